@@ -1,0 +1,159 @@
+/* hpl.h — C ABI of the B200-native NPB-EP hot path (libhpl.so).
+ *
+ * What this library is.  The paper (Bozkus & Fraguela, "A Portable
+ * High-Productivity Approach to Program Heterogeneous Systems", IPDPSW'12)
+ * evaluates HPL — a C++ library whose `Array<T,N>` objects track host and
+ * device copies and whose `eval(f)` runs a
+ * kernel over an index domain — on the NAS EP
+ * benchmark.  This header is the boundary of the
+ * B200 re-design of that hot path: an `Array` coherence layer and a fixed
+ * `eval` of EP, implemented by hand-written sm_100a CUDA kernels.
+ *
+ * Conventions (all functions):
+ *   - extern "C", plain pointers and integers, no C++ or torch types;
+ *   - return an int status (HPL_OK = 0 or a negative HPL_E* code); they never
+ *     throw, abort or exit across the ABI; hpl_last_error() gives detail;
+ *   - outputs are written only when HPL_OK is returned;
+ *   - "device" means the CUDA device current on the calling thread unless a
+ *     device argument says otherwise ("by default the kernel
+ *     is evaluated in the first device found in the system that is not a
+ *     standard general-purpose CPU" — here: the current CUDA device);
+ *   - `stream` arguments are cudaStream_t values passed as void* (NULL = the
+ *     legacy default stream), e.g. torch.cuda.current_stream().cuda_stream.
+ *
+ * EP stream convention (NPB ep.f/randdp.f, the paper's reference [16],
+ * PAPER.md:1322-1323; readings R1-R10):
+ *   x_0 = seed, x_{k+1} = a * x_k mod 2^46, uniform u_j = x_{j+1} * 2^-46,
+ *   pair i = (u_{2i}, u_{2i+1}), x1 = 2u_{2i} - 1, x2 = 2u_{2i+1} - 1,
+ *   t = RN(RN(x1*x1) + RN(x2*x2)); accepted iff t <= 1;
+ *   X = x1*sqrt(-2 ln t / t), Y = x2*sqrt(-2 ln t / t);
+ *   l = trunc(max(|X|,|Y|)), q[l] += 1, sx += X, sy += Y.
+ * Valid parameters: 0 <= M <= 43 (the stream period is 2^44 uniforms),
+ * seed < 2^46 and seed != 2^45, a odd and 1 <= a < 2^46 (reading R9).
+ */
+#ifndef HPL_H_
+#define HPL_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* ---- status codes ------------------------------------------------------ */
+#define HPL_OK 0
+#define HPL_EINVAL (-1)  /* bad argument                                    */
+#define HPL_ENOMEM (-2)  /* host or device allocation failed                */
+#define HPL_ECUDA (-3)   /* CUDA runtime error; detail in hpl_last_error()  */
+#define HPL_ENODEV (-4)  /* no CUDA device / device is not sm_100           */
+#define HPL_ERANGE (-5)  /* an annulus index l >= 10 occurred; result withheld */
+#define HPL_ESTATE (-6)  /* coherence misuse (e.g. data() of an invalid copy) */
+
+/* Static string for a status code (never NULL). */
+const char* hpl_strerror(int code);
+/* Thread-local detail of the last failing call on this thread ("" if none);
+ * valid until the next hpl_* call on the same thread. */
+const char* hpl_last_error(void);
+/* Library ABI version: (major << 16) | minor. */
+int hpl_version(void);
+
+/* ---- devices ----------------------------------------------------------- */
+int hpl_device_count(int* n);
+/* Make `device` current for this thread's subsequent hpl_* calls.  Multi-GPU
+ * callers (one process per GPU) call this with their local rank. */
+int hpl_set_device(int device);
+int hpl_get_device(int* device);
+
+/* ---- Array<T, ndim>: host/device coherence ----------
+ * An hpl_array owns (or borrows) a host copy and owns a device copy of an
+ * ndim-dimensional dense row-major array (ndim 0 = scalar, PAPER.md:361-364;
+ * ndim <= 3 like the paper's index domains).  Two valid bits record which
+ * copies are current; hpl_array_sync() copies only when the requested copy
+ * is stale (the paper's transfer minimisation, PAPER.md:1064-1069,
+ * 1174-1178).  Kernels launched through this library mark their output
+ * arrays device-valid / host-stale. */
+typedef struct hpl_array_s* hpl_array;
+typedef enum { HPL_F64 = 0, HPL_F32 = 1, HPL_U64 = 2, HPL_I64 = 3, HPL_I32 = 4, HPL_U32 = 5 } hpl_dtype;
+typedef enum { HPL_HOST = 1, HPL_DEVICE = 2 } hpl_where;
+typedef enum { HPL_READ = 1, HPL_WRITE = 2, HPL_READWRITE = 3 } hpl_access;
+
+/* Allocate an array of dims[0..ndim-1] elements of type t on `device`
+ * (-1 = current).  host_ptr == NULL: the library allocates a pinned host
+ * buffer and frees it in hpl_array_free; both copies start valid (contents
+ * undefined).  host_ptr != NULL: the caller owns that storage, which must
+ * hold the array and outlive it; the host copy starts
+ * valid and the device copy stale.  Errors: EINVAL (ndim not in 0..3, a dim
+ * <= 0, bad dtype, out == NULL), ENOMEM, ECUDA. */
+int hpl_array_alloc(hpl_array* out, hpl_dtype t, int ndim, const int64_t* dims, void* host_ptr,
+                    int device);
+/* Free the array's device copy and any library-owned host copy.  Pending
+ * work on the array's stream is synchronised first.  NULL is a no-op. */
+int hpl_array_free(hpl_array a);
+/* Make the copy at `where` valid, copying from the other copy only if stale.
+ * mode WRITE or READWRITE additionally invalidates the other copy (the
+ * caller announces it will modify this one).  HOST syncs block until the
+ * data is on the host; DEVICE syncs are stream-ordered on the array stream. */
+int hpl_array_sync(hpl_array a, hpl_where where, hpl_access mode);
+/* Raw pointer to the copy at `where` (the paper's data());
+ * no synchronisation and no validity change. */
+int hpl_array_data(hpl_array a, hpl_where where, void** ptr);
+/* Shape/state query; any output pointer may be NULL.  dims receives ndim
+ * entries.  valid receives a bitmask of HPL_HOST | HPL_DEVICE. */
+int hpl_array_info(hpl_array a, hpl_dtype* t, int* ndim, int64_t* dims, int64_t* nbytes,
+                   int* valid);
+/* Stream used for this array's transfers and for kernels that write it
+ * (NULL = legacy default stream).  The stream must outlive its use. */
+int hpl_array_set_stream(hpl_array a, void* stream);
+
+/* ---- EP: the hot path ----------------------------------------------------
+ * Result layout ("13 words", float64, as exchanged by the multi-GPU
+ * allreduce): [0] sx, [1] sy, [2..11] q[0..9], [12] gc = sum q.  Counts are
+ * exact integers (< 2^53).  If an annulus index l >= 10 occurred (P ~ 1e-22
+ * per pair, never for classes S..E) word [0] is set to NaN and blocking calls
+ * return HPL_ERANGE. */
+
+/* eval(EP) over the 1-D index domain of pairs of shard `rank` of `nranks`
+ * (pairs [rank*2^M/nranks, (rank+1)*2^M/nranks)) into `out13`, an HPL_F64
+ * array with exactly 13 elements, which becomes device-valid/host-stale.
+ * Asynchronous on out13's stream.  nranks must be a power of two <= 2^M. */
+int hpl_ep_eval(int M, uint64_t seed, uint64_t a, int rank, int nranks, hpl_array out13);
+
+/* Whole EP problem of 2^M pairs on the current device; blocking.
+ * sx, sy, q[10] receive the result (gc = sum q). */
+int hpl_ep_run(int M, uint64_t seed, uint64_t a, double* sx, double* sy, uint64_t q[10]);
+
+/* One multi-GPU shard: writes the 13-word partial of pairs
+ * [rank*2^M/nranks, (rank+1)*2^M/nranks) to the caller-owned device buffer
+ * dev_out13 (13 doubles, e.g. a torch tensor), asynchronously on `stream`.
+ * The caller combines shards with one allreduce(SUM). */
+int hpl_ep_run_shard(int M, uint64_t seed, uint64_t a, int rank, int nranks, double* dev_out13,
+                     void* stream);
+
+/* EP over an arbitrary pair range [pair_begin, pair_begin + npairs) of the
+ * stream (npairs may be 0; pair_begin + npairs <= 2^43).  Asynchronous on
+ * `stream`; writes 13 doubles to dev_out13. */
+int hpl_ep_run_range(uint64_t seed, uint64_t a, uint64_t pair_begin, uint64_t npairs,
+                     double* dev_out13, void* stream);
+
+/* Test hook: the LCG states x_{offset+1} .. x_{offset+n} (u64 < 2^46),
+ * computed on the device by the same skip-ahead and step code the EP kernel
+ * uses, copied to host_out[0..n-1].  Blocking.  n <= 2^28. */
+int hpl_lcg_states(uint64_t seed, uint64_t a, uint64_t offset, uint64_t n, uint64_t* host_out);
+
+/* ---- tuning / introspection ------------------------------------------- */
+#define HPL_EP_LEAN 0      /* table log + rsqrt-Newton transform (default)   */
+#define HPL_EP_LIBDEVICE 1 /* CUDA libdevice log / div / sqrt, as NPB writes it */
+/* Select the kernel variant and launch shape for subsequent EP calls on this
+ * thread (threads_per_block 0 / blocks_per_sm 0 = library default). */
+int hpl_ep_set_config(int variant, int threads_per_block, int blocks_per_sm);
+/* Launch shape the library would use for npairs pairs on the current device:
+ * blocks, threads per block, dynamic shared-memory bytes. */
+int hpl_ep_launch_shape(uint64_t npairs, int* blocks, int* threads, int* smem_bytes);
+/* Number of EP kernel launches issued by this process so far (bench.py's
+ * gpu_launches evidence). */
+int hpl_ep_launch_count(uint64_t* count);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* HPL_H_ */

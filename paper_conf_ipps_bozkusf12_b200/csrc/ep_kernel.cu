@@ -1,0 +1,444 @@
+// ep_kernel.cu — the fused NPB-EP hot path for sm_100a.
+//
+// One launch computes the 13-word EP result of a contiguous range of pairs:
+//   A2 per-thread LCG skip-ahead  x = x_begin * a^(2 p0) mod 2^46
+//   A3 uniforms in registers      v = ((a v) & 2^52-1) | bits(1.0)
+//   A4 pair map + acceptance      x1 = 2v-3, t = RN(RN(x1^2)+RN(x2^2)), t <= 1
+//   A5 polar transform            t2 = sqrt(-2 ln t / t)
+//   A6 annulus binning            l = trunc(max(|x1|,|x2|) t2), packed counters
+//   A7 sums                       sx += x1 t2, sy += x2 t2
+//   A8 warp shuffle -> shared-memory block reduction -> per-block partial ->
+//      last-block-done fixed-order finalize into out13 (deterministic).
+// The method is NPB EP (the paper's reference [16]); the
+// stream/acceptance/binning conventions are readings R1-R10 in DESIGN.md.
+// HBM traffic is ~O(grid) bytes; the kernel is FP64-pipe / issue bound.
+#include <cuda_runtime.h>
+
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+#include <vector>
+
+#include "ep_common.cuh"
+#include "ep_launch.h"
+
+namespace hplep {
+
+constexpr int EP_MAX_THREADS = 1024;
+
+__device__ __forceinline__ double as_double(uint64_t v) {
+  return __longlong_as_double(static_cast<long long>(v));
+}
+
+// x * a^k mod 2^46 through the jump table (product of J[i] over set bits of k).
+__device__ __forceinline__ uint64_t jump_state(uint64_t x, uint64_t k, const uint64_t* J) {
+#pragma unroll 1
+  for (int i = 0; i < NJUMP && (k >> i) != 0; ++i)
+    if ((k >> i) & 1) x = mulmod46(x, J[i]);
+  return x;
+}
+
+__device__ __forceinline__ double rsqrt_approx(double p) {
+  double y;
+  asm("rsqrt.approx.ftz.f64 %0, %1;" : "=d"(y) : "d"(p));  // MUFU.RSQ64H, ~2^-20
+  return y;
+}
+
+__device__ __forceinline__ unsigned shl_clamped(unsigned x, unsigned s) {
+  unsigned r;
+  asm("shl.b32 %0, %1, %2;" : "=r"(r) : "r"(x), "r"(s));  // s >= 32 -> 0 (PTX clamps)
+  return r;
+}
+
+template <int VARIANT, bool A32>
+__global__ void __launch_bounds__(EP_MAX_THREADS)
+ep_kernel(const __grid_constant__ EPParams P) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  LogEntry* s_tab = reinterpret_cast<LogEntry*>(smem_raw);
+  __shared__ unsigned long long s_rare[7];  // bins 4..9, then l >= 10
+  __shared__ double s_wsx[EP_MAX_THREADS / 32], s_wsy[EP_MAX_THREADS / 32];
+  __shared__ unsigned long long s_wq[EP_MAX_THREADS / 32][4];
+  __shared__ int s_last;
+  __shared__ double s_fin[13];
+
+  const unsigned tid = threadIdx.x;
+  if (VARIANT == HPL_VARIANT_LEAN) {
+    const double2* src = reinterpret_cast<const double2*>(P.table);
+    double2* dst = reinterpret_cast<double2*>(s_tab);
+    for (unsigned i = tid; i < LOG_N; i += blockDim.x) dst[i] = __ldg(src + i);
+  }
+  if (tid < 7) s_rare[tid] = 0;
+  __syncthreads();
+
+  // ---- A2: this thread's pair range and start state
+  const uint64_t gid = uint64_t(blockIdx.x) * blockDim.x + tid;
+  const uint64_t n_t = P.base + (gid < P.extra ? 1 : 0);
+  const uint64_t p0 = gid * P.base + (gid < P.extra ? gid : P.extra);
+  uint64_t v = state_to_v(jump_state(P.x_begin, 2 * p0, P.jump));
+  const uint64_t a = A32 ? (P.a & 0xFFFFFFFFull) : P.a;
+
+  double sx = 0.0, sy = 0.0;
+  unsigned q0 = 0, q1 = 0, q2 = 0, q3 = 0;
+  uint64_t rem = n_t;
+  while (rem != 0) {
+    // 8-bit packed counters for bins 0..3 overflow after 255 pairs
+    const unsigned chunk = rem < 255 ? unsigned(rem) : 255u;
+    unsigned cnt = 0;
+    double csx = 0.0, csy = 0.0;
+#pragma unroll 4
+    for (unsigned i = 0; i < chunk; ++i) {
+      // ---- A3: two LCG steps; v is the bit pattern of 1 + u
+      v = step_v(v, a);
+      const double v1 = as_double(v);
+      v = step_v(v, a);
+      const double v2 = as_double(v);
+      // ---- A4: x = 2u - 1 = 2v - 3 (exact); t unfused like NPB (R5)
+      const double x1 = fma(v1, 2.0, -3.0);
+      const double x2 = fma(v2, 2.0, -3.0);
+      const double t = __dadd_rn(__dmul_rn(x1, x1), __dmul_rn(x2, x2));
+      const bool acc = t <= 1.0;
+      if (VARIANT == HPL_VARIANT_LIBDEVICE) {
+        // NPB's own formulation: t2 = sqrt(-2 log t / t), X = x1 t2, Y = x2 t2
+        if (acc) {
+          const double t2 = sqrt(-2.0 * log(t) / t);
+          const double X = __dmul_rn(x1, t2), Y = __dmul_rn(x2, t2);
+          const unsigned l = __double2uint_rz(fmax(fabs(X), fabs(Y)));
+          csx += X;
+          csy += Y;
+          cnt += shl_clamped(1u, l << 3);
+          if (l >= 4) atomicAdd(&s_rare[(l < 10 ? l : 10u) - 4], 1ull);
+        }
+      } else {
+        // ---- A5 lean: L = -2 ln t = T[u] + r q(r) (table + degree-6 series)
+        const unsigned H = static_cast<unsigned>(__double2hiint(t));
+        const unsigned u = (H + LOG_ADD) >> LOG_SHIFT;
+        const unsigned uc = u < LOG_N ? u : LOG_N - 1;
+        const double2 ent = reinterpret_cast<const double2*>(s_tab)[uc];
+        const double r = fma(t, ent.y, -1.0);
+        double c = fma(1.0 / 3.0, r, -0.4);
+        c = fma(c, r, 0.5);
+        c = fma(c, r, -2.0 / 3.0);
+        c = fma(c, r, 1.0);
+        c = fma(c, r, -2.0);
+        double L = fma(c, r, ent.x);
+        if (acc && u >= LOG_N) L = -2.0 * log(t);  // t < 2^-16: rare slow path
+        // t2 = sqrt(L / t) = L * rsqrt(L t); one cubic Newton step from MUFU
+        const double p = fma(L, t, 0x1p-200);  // + tiny: t == 1 gives L = 0 -> t2 = 0
+        const double y0 = rsqrt_approx(p);
+        const double h = __dmul_rn(p, y0);
+        const double e = fma(-h, y0, 1.0);
+        const double cc = fma(e, 0.375, 0.5);
+        const double g = __dmul_rn(L, y0);
+        const double ge = __dmul_rn(g, e);
+        const double t2 = fma(ge, cc, g);
+        // ---- A6: l = trunc(RN(max(|x1|,|x2|) t2)) == trunc(max(|X|,|Y|))
+        const double mm = __dmul_rn(fmax(fabs(x1), fabs(x2)), t2);
+        const unsigned l = __double2uint_rz(mm);
+        if (acc) {
+          // ---- A7
+          csx = fma(x1, t2, csx);
+          csy = fma(x2, t2, csy);
+          cnt += shl_clamped(1u, l << 3);
+          if (l >= 4) atomicAdd(&s_rare[(l < 10 ? l : 10u) - 4], 1ull);
+        }
+      }
+    }
+    q0 += cnt & 0xFFu;
+    q1 += (cnt >> 8) & 0xFFu;
+    q2 += (cnt >> 16) & 0xFFu;
+    q3 += cnt >> 24;
+    sx += csx;
+    sy += csy;
+    rem -= chunk;
+  }
+
+  // ---- A8: warp -> block reduction (fixed order => deterministic)
+  unsigned long long w0 = q0, w1 = q1, w2 = q2, w3 = q3;
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) {
+    sx += __shfl_xor_sync(0xFFFFFFFFu, sx, off);
+    sy += __shfl_xor_sync(0xFFFFFFFFu, sy, off);
+    w0 += __shfl_xor_sync(0xFFFFFFFFu, w0, off);
+    w1 += __shfl_xor_sync(0xFFFFFFFFu, w1, off);
+    w2 += __shfl_xor_sync(0xFFFFFFFFu, w2, off);
+    w3 += __shfl_xor_sync(0xFFFFFFFFu, w3, off);
+  }
+  const unsigned warp = tid >> 5, lane = tid & 31;
+  if (lane == 0) {
+    s_wsx[warp] = sx;
+    s_wsy[warp] = sy;
+    s_wq[warp][0] = w0;
+    s_wq[warp][1] = w1;
+    s_wq[warp][2] = w2;
+    s_wq[warp][3] = w3;
+  }
+  __syncthreads();
+  if (tid == 0) {
+    EPPartial part;
+    part.sx = 0.0;
+    part.sy = 0.0;
+    for (int k = 0; k < 4; ++k) part.q[k] = 0;
+    const unsigned nw = blockDim.x >> 5;
+    for (unsigned w = 0; w < nw; ++w) {
+      part.sx += s_wsx[w];
+      part.sy += s_wsy[w];
+      for (int k = 0; k < 4; ++k) part.q[k] += s_wq[w][k];
+    }
+    for (int k = 4; k < 10; ++k) part.q[k] = s_rare[k - 4];
+    part.big = s_rare[6];
+    P.partials[blockIdx.x] = part;
+    __threadfence();
+    const unsigned ticket = atomicAdd(P.counter, 1u);
+    s_last = (ticket == gridDim.x - 1);
+  }
+  __syncthreads();
+  if (!s_last) return;
+  // last block: word w of the result summed over blocks 0..G-1 in order
+  __threadfence();
+  if (tid < 13) {
+    const unsigned G = gridDim.x;
+    if (tid < 2) {
+      double s = 0.0;
+      for (unsigned b = 0; b < G; ++b) s += __ldcg(tid == 0 ? &P.partials[b].sx : &P.partials[b].sy);
+      s_fin[tid] = s;
+    } else {
+      unsigned long long s = 0;
+      for (unsigned b = 0; b < G; ++b)
+        s += __ldcg(tid < 12 ? &P.partials[b].q[tid - 2] : &P.partials[b].big);
+      s_fin[tid] = static_cast<double>(s);  // exact: < 2^53
+    }
+  }
+  __syncthreads();
+  if (tid == 0) {
+    double gc = 0.0;
+    for (int k = 0; k < 10; ++k) gc += s_fin[2 + k];  // exact integer sum
+    const bool big = s_fin[12] != 0.0;
+    P.out13[0] = big ? __longlong_as_double(0x7FF8000000000000ll) : s_fin[0];
+    P.out13[1] = s_fin[1];
+    for (int k = 0; k < 10; ++k) P.out13[2 + k] = s_fin[2 + k];
+    P.out13[12] = gc;
+    *P.counter = 0;  // ready for the next launch on this workspace
+  }
+}
+
+// Test hook kernel: x_{offset+i+1} via the kernel's own jump + step code.
+__global__ void lcg_states_kernel(uint64_t seed, uint64_t a, uint64_t offset, uint64_t n,
+                                  const __grid_constant__ JumpTable J, uint64_t* out) {
+  const uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  uint64_t v = state_to_v(jump_state(seed, offset + i, J.j));
+  v = step_v(v, a);
+  out[i] = v_to_state(v);
+}
+
+// ------------------------------------------------------------------ host side
+void build_jump_table(uint64_t a, uint64_t* J) {
+  uint64_t x = a & MASK46;
+  for (int i = 0; i < NJUMP; ++i) {
+    J[i] = x;
+    x = mulmod46(x, x);
+  }
+}
+
+uint64_t host_jump(uint64_t x, uint64_t k, const uint64_t* J) {
+  for (int i = 0; i < NJUMP && (k >> i) != 0; ++i)
+    if ((k >> i) & 1) x = mulmod46(x, J[i]);
+  return x;
+}
+
+// Lean-log table, built in 80-bit long double on the host.
+void build_log_table(std::vector<LogEntry>& tab) {
+  tab.resize(LOG_N);
+  for (uint32_t u = 0; u < LOG_N; ++u) {
+    const uint32_t idx = LOG_IDX_MIN + u;
+    const int E = int(idx >> LOG_K) - 1023;
+    const long double centre = ldexpl(1.0L + (long double)(idx & ((1u << LOG_K) - 1)) / (1 << LOG_K), E);
+    const float inv = (float)(1.0L / centre);
+    tab[u].inv = (double)inv;
+    tab[u].T = (double)(2.0L * logl((long double)inv));
+  }
+}
+
+namespace {
+struct DeviceState {
+  LogEntry* table = nullptr;
+  int sms = 0;
+  int max_smem_optin = 0;
+};
+std::mutex g_mu;
+std::vector<DeviceState> g_dev;
+struct Workspace {
+  int device;
+  cudaStream_t stream;
+  EPPartial* partials;
+  unsigned* counter;
+  int capacity;
+};
+std::vector<Workspace> g_ws;
+unsigned long long g_launches = 0;
+
+int set_attrs_once(int device) {
+  static std::vector<char> done;
+  if ((int)done.size() <= device) done.resize(device + 1, 0);
+  if (done[device]) return 0;
+  const int smem = int(LOG_N * sizeof(LogEntry));
+  cudaError_t e;
+  e = cudaFuncSetAttribute(ep_kernel<HPL_VARIANT_LEAN, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(ep_kernel<HPL_VARIANT_LEAN, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e != cudaSuccess) return set_cuda_error(e, "cudaFuncSetAttribute");
+  done[device] = 1;
+  return 0;
+}
+}  // namespace
+
+int device_state(int device, const LogEntry** table, int* sms) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  if ((int)g_dev.size() <= device) g_dev.resize(device + 1);
+  DeviceState& d = g_dev[device];
+  if (d.table == nullptr) {
+    cudaDeviceProp prop;
+    cudaError_t e = cudaGetDeviceProperties(&prop, device);
+    if (e != cudaSuccess) return set_cuda_error(e, "cudaGetDeviceProperties");
+    if (prop.major != 10) return set_error(HPL_ENODEV, "device is sm_%d%d, this build targets sm_100a", prop.major, prop.minor);
+    d.sms = prop.multiProcessorCount;
+    d.max_smem_optin = int(prop.sharedMemPerBlockOptin);
+    std::vector<LogEntry> tab;
+    build_log_table(tab);
+    LogEntry* dt = nullptr;
+    e = cudaMalloc(&dt, tab.size() * sizeof(LogEntry));
+    if (e != cudaSuccess) return set_cuda_error(e, "cudaMalloc(log table)");
+    e = cudaMemcpy(dt, tab.data(), tab.size() * sizeof(LogEntry), cudaMemcpyHostToDevice);
+    if (e != cudaSuccess) { cudaFree(dt); return set_cuda_error(e, "cudaMemcpy(log table)"); }
+    d.table = dt;
+    int rc = set_attrs_once(device);
+    if (rc) return rc;
+  }
+  *table = d.table;
+  *sms = d.sms;
+  return 0;
+}
+
+static int workspace(int device, cudaStream_t stream, int blocks, EPPartial** partials, unsigned** counter) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  for (auto& w : g_ws) {
+    if (w.device == device && w.stream == stream) {
+      if (w.capacity < blocks) {
+        cudaError_t e = cudaStreamSynchronize(stream);
+        if (e != cudaSuccess) return set_cuda_error(e, "cudaStreamSynchronize");
+        cudaFree(w.partials);
+        w.partials = nullptr;
+        e = cudaMalloc(&w.partials, sizeof(EPPartial) * blocks);
+        if (e != cudaSuccess) return set_cuda_error(e, "cudaMalloc(partials)");
+        w.capacity = blocks;
+      }
+      *partials = w.partials;
+      *counter = w.counter;
+      return 0;
+    }
+  }
+  Workspace w{device, stream, nullptr, nullptr, blocks};
+  cudaError_t e = cudaMalloc(&w.partials, sizeof(EPPartial) * blocks);
+  if (e != cudaSuccess) return set_cuda_error(e, "cudaMalloc(partials)");
+  e = cudaMalloc(&w.counter, sizeof(unsigned));
+  if (e == cudaSuccess) e = cudaMemset(w.counter, 0, sizeof(unsigned));
+  if (e != cudaSuccess) { cudaFree(w.partials); return set_cuda_error(e, "cudaMalloc(counter)"); }
+  g_ws.push_back(w);
+  *partials = w.partials;
+  *counter = w.counter;
+  return 0;
+}
+
+int launch_shape(int device, uint64_t npairs, const EPConfig& cfg, int* blocks, int* threads, int* smem) {
+  const LogEntry* tab;
+  int sms;
+  int rc = device_state(device, &tab, &sms);
+  if (rc) return rc;
+  const int thr = cfg.threads_per_block > 0 ? cfg.threads_per_block : EP_DEFAULT_THREADS;
+  if (thr < 32 || thr > EP_MAX_THREADS || thr % 32) return set_error(HPL_EINVAL, "threads_per_block must be a multiple of 32 in [32, 1024]");
+  const int sm_bytes = cfg.variant == HPL_VARIANT_LEAN ? int(LOG_N * sizeof(LogEntry)) : 0;
+  int bps = cfg.blocks_per_sm;
+  if (bps <= 0) {
+    int occ = 0;
+    cudaError_t e = cfg.variant == HPL_VARIANT_LEAN
+        ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ep_kernel<HPL_VARIANT_LEAN, true>, thr, sm_bytes)
+        : cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ep_kernel<HPL_VARIANT_LIBDEVICE, true>, thr, 0);
+    if (e != cudaSuccess) return set_cuda_error(e, "cudaOccupancyMaxActiveBlocksPerMultiprocessor");
+    bps = occ > 0 ? occ : 1;
+  }
+  // at least EP_MIN_PAIRS_PER_THREAD pairs per thread so skip-ahead stays negligible
+  uint64_t want = (npairs + uint64_t(thr) * EP_MIN_PAIRS_PER_THREAD - 1) / (uint64_t(thr) * EP_MIN_PAIRS_PER_THREAD);
+  uint64_t full = uint64_t(sms) * bps;
+  uint64_t b = want < full ? want : full;
+  if (b < 1) b = 1;
+  *blocks = int(b);
+  *threads = thr;
+  *smem = sm_bytes;
+  return 0;
+}
+
+int launch_ep(int device, uint64_t seed, uint64_t a, uint64_t pair_begin, uint64_t npairs,
+              const EPConfig& cfg, double* dev_out13, cudaStream_t stream) {
+  const LogEntry* tab;
+  int sms;
+  int rc = device_state(device, &tab, &sms);
+  if (rc) return rc;
+  int blocks, threads, smem;
+  rc = launch_shape(device, npairs, cfg, &blocks, &threads, &smem);
+  if (rc) return rc;
+  EPPartial* partials;
+  unsigned* counter;
+  rc = workspace(device, stream, blocks, &partials, &counter);
+  if (rc) return rc;
+
+  EPParams P;
+  std::memset(&P, 0, sizeof(P));
+  build_jump_table(a, P.jump);
+  P.a = a;
+  P.x_begin = host_jump(seed & MASK46, 2 * pair_begin, P.jump);
+  P.npairs = npairs;
+  const uint64_t T = uint64_t(blocks) * threads;
+  P.base = npairs / T;
+  P.extra = npairs % T;
+  P.table = tab;
+  P.partials = partials;
+  P.counter = counter;
+  P.out13 = dev_out13;
+
+  const bool a32 = (a >> 32) == 0;
+  if (cfg.variant == HPL_VARIANT_LEAN) {
+    if (a32) ep_kernel<HPL_VARIANT_LEAN, true><<<blocks, threads, smem, stream>>>(P);
+    else ep_kernel<HPL_VARIANT_LEAN, false><<<blocks, threads, smem, stream>>>(P);
+  } else {
+    if (a32) ep_kernel<HPL_VARIANT_LIBDEVICE, true><<<blocks, threads, 0, stream>>>(P);
+    else ep_kernel<HPL_VARIANT_LIBDEVICE, false><<<blocks, threads, 0, stream>>>(P);
+  }
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return set_cuda_error(e, "ep_kernel launch");
+  {
+    std::lock_guard<std::mutex> lk(g_mu);
+    ++g_launches;
+  }
+  return 0;
+}
+
+unsigned long long launch_count() {
+  std::lock_guard<std::mutex> lk(g_mu);
+  return g_launches;
+}
+
+int launch_lcg_states(uint64_t seed, uint64_t a, uint64_t offset, uint64_t n, uint64_t* dev_out,
+                      cudaStream_t stream) {
+  JumpTable J;
+  build_jump_table(a, J.j);
+  const int thr = 256;
+  const uint64_t blocks = (n + thr - 1) / thr;
+  if (blocks == 0) return 0;
+  lcg_states_kernel<<<unsigned(blocks), thr, 0, stream>>>(seed & MASK46, a, offset, n, J, dev_out);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return set_cuda_error(e, "lcg_states_kernel launch");
+  return 0;
+}
+
+}  // namespace hplep

@@ -1,0 +1,42 @@
+// ep_launch.h — internal interface between the C ABI (hpl_runtime.cpp) and the
+// EP kernels (ep_kernel.cu).  Not installed; include/hpl.h is the public API.
+#pragma once
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "../../include/hpl.h"
+#include "ep_common.cuh"
+
+namespace hplep {
+
+constexpr int HPL_VARIANT_LEAN = HPL_EP_LEAN;
+constexpr int HPL_VARIANT_LIBDEVICE = HPL_EP_LIBDEVICE;
+constexpr int EP_DEFAULT_THREADS = 512;
+constexpr uint64_t EP_MIN_PAIRS_PER_THREAD = 64;
+
+struct EPConfig {
+  int variant = HPL_VARIANT_LEAN;
+  int threads_per_block = 0;  // 0 = EP_DEFAULT_THREADS
+  int blocks_per_sm = 0;      // 0 = occupancy-derived
+};
+
+struct JumpTable {
+  uint64_t j[NJUMP];
+};
+
+// error plumbing (hpl_runtime.cpp): record detail, return the code
+int set_error(int code, const char* fmt, ...);
+int set_cuda_error(cudaError_t e, const char* what);
+
+void build_jump_table(uint64_t a, uint64_t* J);
+uint64_t host_jump(uint64_t x, uint64_t k, const uint64_t* J);
+
+int launch_shape(int device, uint64_t npairs, const EPConfig& cfg, int* blocks, int* threads, int* smem);
+int launch_ep(int device, uint64_t seed, uint64_t a, uint64_t pair_begin, uint64_t npairs,
+              const EPConfig& cfg, double* dev_out13, cudaStream_t stream);
+int launch_lcg_states(uint64_t seed, uint64_t a, uint64_t offset, uint64_t n, uint64_t* dev_out,
+                      cudaStream_t stream);
+unsigned long long launch_count();
+
+}  // namespace hplep

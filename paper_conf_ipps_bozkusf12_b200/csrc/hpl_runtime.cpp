@@ -1,0 +1,373 @@
+// hpl_runtime.cpp — the C ABI declared in include/hpl.h: error plumbing,
+// devices, the Array coherence layer (PAPER.md:331-381, 1064-1069,
+// 1174-1178) and the EP entry points (argument validation, sharding,
+// result delivery).  All compute runs in ep_kernel.cu; nothing here computes
+// any step of EP on the host.
+#include <cuda_runtime.h>
+
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <string>
+
+#include "../../include/hpl.h"
+#include "ep_launch.h"
+
+namespace hplep {
+
+namespace {
+thread_local std::string t_err;
+thread_local EPConfig t_cfg;
+}  // namespace
+
+int set_error(int code, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  t_err = buf;
+  return code;
+}
+
+int set_cuda_error(cudaError_t e, const char* what) {
+  cudaGetLastError();  // clear a non-sticky error
+  if (e == cudaErrorNoDevice || e == cudaErrorInsufficientDriver)
+    return set_error(HPL_ENODEV, "%s: %s", what, cudaGetErrorString(e));
+  if (e == cudaErrorMemoryAllocation) return set_error(HPL_ENOMEM, "%s: %s", what, cudaGetErrorString(e));
+  return set_error(HPL_ECUDA, "%s: %s", what, cudaGetErrorString(e));
+}
+
+static int current_device(int* dev) {
+  cudaError_t e = cudaGetDevice(dev);
+  if (e != cudaSuccess) return set_cuda_error(e, "cudaGetDevice");
+  return 0;
+}
+
+// reading R9: odd a < 2^46, seed < 2^46, seed != 2^45 (the fixed point that
+// would give t = 0); M <= 43 because the stream period is 2^44 uniforms.
+static int validate(uint64_t seed, uint64_t a) {
+  if (seed >> 46) return set_error(HPL_EINVAL, "seed must be < 2^46");
+  if (seed == (uint64_t(1) << 45)) return set_error(HPL_EINVAL, "seed = 2^45 is a fixed point (x1 = x2 = 0, log 0)");
+  if ((a >> 46) || (a & 1) == 0) return set_error(HPL_EINVAL, "a must be odd and < 2^46");
+  return 0;
+}
+
+static int shard_range(int M, int rank, int nranks, uint64_t* begin, uint64_t* n) {
+  if (M < 0 || M > 43) return set_error(HPL_EINVAL, "M must be in [0, 43] (period 2^44)");
+  if (nranks < 1 || (nranks & (nranks - 1)) || uint64_t(nranks) > (uint64_t(1) << M))
+    return set_error(HPL_EINVAL, "nranks must be a power of two <= 2^M");
+  if (rank < 0 || rank >= nranks) return set_error(HPL_EINVAL, "rank out of range");
+  *n = (uint64_t(1) << M) / uint64_t(nranks);
+  *begin = uint64_t(rank) * (*n);
+  return 0;
+}
+
+}  // namespace hplep
+
+using namespace hplep;
+
+struct hpl_array_s {
+  hpl_dtype t;
+  int ndim;
+  int64_t dims[3];
+  int64_t count;
+  size_t nbytes;
+  void* host;
+  bool host_owned;
+  void* dev;
+  int device;
+  cudaStream_t stream;
+  int valid;
+};
+
+static size_t dtype_size(int t) {
+  switch (t) {
+    case HPL_F64: case HPL_U64: case HPL_I64: return 8;
+    case HPL_F32: case HPL_I32: case HPL_U32: return 4;
+    default: return 0;
+  }
+}
+
+namespace {
+struct DeviceGuard {  // make `dev` current for the scope, restore afterwards
+  int prev = -1;
+  int rc = 0;
+  explicit DeviceGuard(int dev) {
+    cudaError_t e = cudaGetDevice(&prev);
+    if (e == cudaSuccess && prev != dev) e = cudaSetDevice(dev);
+    if (e != cudaSuccess) rc = set_cuda_error(e, "cudaSetDevice");
+  }
+  ~DeviceGuard() {
+    int cur;
+    if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+  }
+};
+}  // namespace
+
+extern "C" {
+
+const char* hpl_strerror(int code) {
+  switch (code) {
+    case HPL_OK: return "success";
+    case HPL_EINVAL: return "invalid argument";
+    case HPL_ENOMEM: return "out of memory";
+    case HPL_ECUDA: return "CUDA error";
+    case HPL_ENODEV: return "no suitable CUDA device";
+    case HPL_ERANGE: return "annulus index out of range (l >= 10)";
+    case HPL_ESTATE: return "array coherence misuse";
+    default: return "unknown status";
+  }
+}
+
+const char* hpl_last_error(void) { return t_err.c_str(); }
+
+int hpl_version(void) { return (1 << 16) | 0; }
+
+int hpl_device_count(int* n) {
+  if (!n) return set_error(HPL_EINVAL, "n is NULL");
+  int c = 0;
+  cudaError_t e = cudaGetDeviceCount(&c);
+  if (e != cudaSuccess) return set_cuda_error(e, "cudaGetDeviceCount");
+  *n = c;
+  return HPL_OK;
+}
+
+int hpl_set_device(int device) {
+  int n = 0;
+  int rc = hpl_device_count(&n);
+  if (rc) return rc;
+  if (device < 0 || device >= n) return set_error(HPL_EINVAL, "device %d out of range [0, %d)", device, n);
+  cudaError_t e = cudaSetDevice(device);
+  if (e != cudaSuccess) return set_cuda_error(e, "cudaSetDevice");
+  return HPL_OK;
+}
+
+int hpl_get_device(int* device) {
+  if (!device) return set_error(HPL_EINVAL, "device is NULL");
+  return current_device(device);
+}
+
+// ------------------------------------------------------------------ arrays
+int hpl_array_alloc(hpl_array* out, hpl_dtype t, int ndim, const int64_t* dims, void* host_ptr,
+                    int device) {
+  if (!out) return set_error(HPL_EINVAL, "out is NULL");
+  const size_t es = dtype_size(t);
+  if (es == 0) return set_error(HPL_EINVAL, "bad dtype %d", (int)t);
+  if (ndim < 0 || ndim > 3) return set_error(HPL_EINVAL, "ndim must be in [0, 3]");
+  if (ndim > 0 && !dims) return set_error(HPL_EINVAL, "dims is NULL");
+  int64_t count = 1;
+  for (int i = 0; i < ndim; ++i) {
+    if (dims[i] <= 0) return set_error(HPL_EINVAL, "dims[%d] = %lld must be > 0", i, (long long)dims[i]);
+    if (count > (int64_t(1) << 50) / dims[i]) return set_error(HPL_EINVAL, "array too large");
+    count *= dims[i];
+  }
+  if (device < 0) {
+    int rc = current_device(&device);
+    if (rc) return rc;
+  }
+  int ndev = 0;
+  int rc = hpl_device_count(&ndev);
+  if (rc) return rc;
+  if (device >= ndev) return set_error(HPL_EINVAL, "device %d out of range", device);
+  DeviceGuard g(device);
+  if (g.rc) return g.rc;
+  hpl_array a = new (std::nothrow) hpl_array_s();
+  if (!a) return set_error(HPL_ENOMEM, "host allocation of the descriptor");
+  a->t = t;
+  a->ndim = ndim;
+  for (int i = 0; i < 3; ++i) a->dims[i] = i < ndim ? dims[i] : 1;
+  a->count = count;
+  a->nbytes = size_t(count) * es;
+  a->device = device;
+  a->stream = nullptr;
+  cudaError_t e = cudaMalloc(&a->dev, a->nbytes);
+  if (e != cudaSuccess) { delete a; return set_cuda_error(e, "cudaMalloc(array)"); }
+  if (host_ptr) {
+    a->host = host_ptr;
+    a->host_owned = false;
+    a->valid = HPL_HOST;
+  } else {
+    e = cudaMallocHost(&a->host, a->nbytes);
+    if (e != cudaSuccess) { cudaFree(a->dev); delete a; return set_cuda_error(e, "cudaMallocHost(array)"); }
+    a->host_owned = true;
+    a->valid = HPL_HOST | HPL_DEVICE;
+  }
+  *out = a;
+  return HPL_OK;
+}
+
+int hpl_array_free(hpl_array a) {
+  if (!a) return HPL_OK;
+  DeviceGuard g(a->device);
+  cudaError_t e1 = a->stream ? cudaStreamSynchronize(a->stream) : cudaDeviceSynchronize();
+  cudaError_t e2 = cudaFree(a->dev);
+  cudaError_t e3 = a->host_owned ? cudaFreeHost(a->host) : cudaSuccess;
+  delete a;
+  if (e1 != cudaSuccess) return set_cuda_error(e1, "hpl_array_free: synchronize");
+  if (e2 != cudaSuccess) return set_cuda_error(e2, "cudaFree");
+  if (e3 != cudaSuccess) return set_cuda_error(e3, "cudaFreeHost");
+  return HPL_OK;
+}
+
+int hpl_array_sync(hpl_array a, hpl_where where, hpl_access mode) {
+  if (!a) return set_error(HPL_EINVAL, "array is NULL");
+  if (where != HPL_HOST && where != HPL_DEVICE) return set_error(HPL_EINVAL, "bad where");
+  if (mode < HPL_READ || mode > HPL_READWRITE) return set_error(HPL_EINVAL, "bad access mode");
+  DeviceGuard g(a->device);
+  if (g.rc) return g.rc;
+  if (!(a->valid & where)) {
+    if (!(a->valid & (where == HPL_HOST ? HPL_DEVICE : HPL_HOST)))
+      return set_error(HPL_ESTATE, "neither copy is valid");
+    cudaError_t e;
+    if (where == HPL_HOST) {
+      e = cudaMemcpyAsync(a->host, a->dev, a->nbytes, cudaMemcpyDeviceToHost, a->stream);
+      if (e == cudaSuccess) e = cudaStreamSynchronize(a->stream);
+    } else {
+      e = cudaMemcpyAsync(a->dev, a->host, a->nbytes, cudaMemcpyHostToDevice, a->stream);
+    }
+    if (e != cudaSuccess) return set_cuda_error(e, "hpl_array_sync copy");
+    a->valid |= where;
+  } else if (where == HPL_HOST && (mode & HPL_WRITE) && (a->valid & HPL_DEVICE)) {
+    // the host is about to be modified while device work may still read it
+    cudaError_t e = cudaStreamSynchronize(a->stream);
+    if (e != cudaSuccess) return set_cuda_error(e, "hpl_array_sync synchronize");
+  }
+  if (mode & HPL_WRITE) a->valid = where;
+  return HPL_OK;
+}
+
+int hpl_array_data(hpl_array a, hpl_where where, void** ptr) {
+  if (!a || !ptr) return set_error(HPL_EINVAL, "NULL argument");
+  if (where == HPL_HOST) *ptr = a->host;
+  else if (where == HPL_DEVICE) *ptr = a->dev;
+  else return set_error(HPL_EINVAL, "bad where");
+  return HPL_OK;
+}
+
+int hpl_array_info(hpl_array a, hpl_dtype* t, int* ndim, int64_t* dims, int64_t* nbytes, int* valid) {
+  if (!a) return set_error(HPL_EINVAL, "array is NULL");
+  if (t) *t = a->t;
+  if (ndim) *ndim = a->ndim;
+  if (dims) for (int i = 0; i < a->ndim; ++i) dims[i] = a->dims[i];
+  if (nbytes) *nbytes = int64_t(a->nbytes);
+  if (valid) *valid = a->valid;
+  return HPL_OK;
+}
+
+int hpl_array_set_stream(hpl_array a, void* stream) {
+  if (!a) return set_error(HPL_EINVAL, "array is NULL");
+  a->stream = static_cast<cudaStream_t>(stream);
+  return HPL_OK;
+}
+
+// --------------------------------------------------------------------- EP
+int hpl_ep_run_range(uint64_t seed, uint64_t a, uint64_t pair_begin, uint64_t npairs,
+                     double* dev_out13, void* stream) {
+  int rc = validate(seed, a);
+  if (rc) return rc;
+  if (!dev_out13) return set_error(HPL_EINVAL, "dev_out13 is NULL");
+  if (pair_begin > (uint64_t(1) << 43) || npairs > (uint64_t(1) << 43) - pair_begin)
+    return set_error(HPL_EINVAL, "pair range beyond 2^43 (period 2^44 uniforms)");
+  int dev;
+  rc = current_device(&dev);
+  if (rc) return rc;
+  return launch_ep(dev, seed, a, pair_begin, npairs, t_cfg, dev_out13, static_cast<cudaStream_t>(stream));
+}
+
+int hpl_ep_run_shard(int M, uint64_t seed, uint64_t a, int rank, int nranks, double* dev_out13,
+                     void* stream) {
+  uint64_t begin, n;
+  int rc = shard_range(M, rank, nranks, &begin, &n);
+  if (rc) return rc;
+  return hpl_ep_run_range(seed, a, begin, n, dev_out13, stream);
+}
+
+int hpl_ep_eval(int M, uint64_t seed, uint64_t a, int rank, int nranks, hpl_array out13) {
+  if (!out13) return set_error(HPL_EINVAL, "out13 is NULL");
+  if (out13->t != HPL_F64 || out13->count != 13) return set_error(HPL_EINVAL, "out13 must be an HPL_F64 array of 13 elements");
+  uint64_t begin, n;
+  int rc = shard_range(M, rank, nranks, &begin, &n);
+  if (rc) return rc;
+  rc = validate(seed, a);
+  if (rc) return rc;
+  DeviceGuard g(out13->device);
+  if (g.rc) return g.rc;
+  rc = launch_ep(out13->device, seed, a, begin, n, t_cfg, static_cast<double*>(out13->dev), out13->stream);
+  if (rc) return rc;
+  out13->valid = HPL_DEVICE;  // the kernel wrote the device copy
+  return HPL_OK;
+}
+
+int hpl_ep_run(int M, uint64_t seed, uint64_t a, double* sx, double* sy, uint64_t q[10]) {
+  if (!sx || !sy || !q) return set_error(HPL_EINVAL, "NULL output pointer");
+  int dev;
+  int rc = current_device(&dev);
+  if (rc) return rc;
+  // one cached 13-word Array per thread and device (the paper's Array with
+  // a library-owned host copy)
+  thread_local hpl_array cache[64] = {nullptr};
+  if (dev >= 64) return set_error(HPL_EINVAL, "device index too large");
+  if (!cache[dev]) {
+    int64_t d = 13;
+    rc = hpl_array_alloc(&cache[dev], HPL_F64, 1, &d, nullptr, dev);
+    if (rc) return rc;
+  }
+  hpl_array out = cache[dev];
+  rc = hpl_ep_eval(M, seed, a, 0, 1, out);
+  if (rc) return rc;
+  rc = hpl_array_sync(out, HPL_HOST, HPL_READ);  // 104-byte D2H, blocking
+  if (rc) return rc;
+  const double* h = static_cast<const double*>(out->host);
+  if (h[0] != h[0]) return set_error(HPL_ERANGE, "an annulus index l >= 10 occurred");
+  *sx = h[0];
+  *sy = h[1];
+  for (int k = 0; k < 10; ++k) q[k] = static_cast<uint64_t>(h[2 + k]);
+  return HPL_OK;
+}
+
+int hpl_lcg_states(uint64_t seed, uint64_t a, uint64_t offset, uint64_t n, uint64_t* host_out) {
+  int rc = validate(seed, a);
+  if (rc) return rc;
+  if (n > (uint64_t(1) << 28)) return set_error(HPL_EINVAL, "n must be <= 2^28");
+  if (n == 0) return HPL_OK;
+  if (!host_out) return set_error(HPL_EINVAL, "host_out is NULL");
+  uint64_t* d = nullptr;
+  cudaError_t e = cudaMalloc(&d, n * sizeof(uint64_t));
+  if (e != cudaSuccess) return set_cuda_error(e, "cudaMalloc(states)");
+  rc = launch_lcg_states(seed, a, offset, n, d, nullptr);
+  if (!rc) {
+    e = cudaMemcpy(host_out, d, n * sizeof(uint64_t), cudaMemcpyDeviceToHost);
+    if (e != cudaSuccess) rc = set_cuda_error(e, "cudaMemcpy(states)");
+  }
+  cudaFree(d);
+  return rc;
+}
+
+int hpl_ep_set_config(int variant, int threads_per_block, int blocks_per_sm) {
+  if (variant != HPL_EP_LEAN && variant != HPL_EP_LIBDEVICE) return set_error(HPL_EINVAL, "unknown variant");
+  if (threads_per_block < 0 || threads_per_block > 1024 || threads_per_block % 32)
+    return set_error(HPL_EINVAL, "threads_per_block must be 0 or a multiple of 32 <= 1024");
+  if (blocks_per_sm < 0 || blocks_per_sm > 32) return set_error(HPL_EINVAL, "blocks_per_sm must be in [0, 32]");
+  t_cfg.variant = variant;
+  t_cfg.threads_per_block = threads_per_block;
+  t_cfg.blocks_per_sm = blocks_per_sm;
+  return HPL_OK;
+}
+
+int hpl_ep_launch_shape(uint64_t npairs, int* blocks, int* threads, int* smem_bytes) {
+  if (!blocks || !threads || !smem_bytes) return set_error(HPL_EINVAL, "NULL output pointer");
+  int dev;
+  int rc = current_device(&dev);
+  if (rc) return rc;
+  return launch_shape(dev, npairs, t_cfg, blocks, threads, smem_bytes);
+}
+
+int hpl_ep_launch_count(uint64_t* count) {
+  if (!count) return set_error(HPL_EINVAL, "count is NULL");
+  *count = launch_count();
+  return HPL_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,211 @@
+"""Thin ctypes binding of include/hpl.h (libhpl.so) — argument marshalling only.
+
+Every step of EP runs in the CUDA kernels of ``csrc/``; nothing here computes.
+If ``libhpl.so`` is missing the import fails loudly (no CPU fallback): build it
+with ``python -m paper_conf_ipps_bozkusf12_b200.build`` (or
+``__graft_entry__.build()``).
+
+Names mirror the C ABI: ``hpl_array_alloc``, ``hpl_array_sync``,
+``hpl_ep_run``, ``hpl_ep_run_shard``, ... .  Functions raise :class:`HPLError`
+on a non-zero status; the C status code is ``err.code``.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libhpl.so")
+
+HPL_OK, HPL_EINVAL, HPL_ENOMEM, HPL_ECUDA, HPL_ENODEV, HPL_ERANGE, HPL_ESTATE = 0, -1, -2, -3, -4, -5, -6
+HPL_F64, HPL_F32, HPL_U64, HPL_I64, HPL_I32, HPL_U32 = 0, 1, 2, 3, 4, 5
+HPL_HOST, HPL_DEVICE = 1, 2
+HPL_READ, HPL_WRITE, HPL_READWRITE = 1, 2, 3
+HPL_EP_LEAN, HPL_EP_LIBDEVICE = 0, 1
+
+# every symbol include/hpl.h declares (tests/test_abi.py checks the header agrees)
+EXPORTS = (
+    "hpl_strerror", "hpl_last_error", "hpl_version",
+    "hpl_device_count", "hpl_set_device", "hpl_get_device",
+    "hpl_array_alloc", "hpl_array_free", "hpl_array_sync", "hpl_array_data",
+    "hpl_array_info", "hpl_array_set_stream",
+    "hpl_ep_eval", "hpl_ep_run", "hpl_ep_run_shard", "hpl_ep_run_range",
+    "hpl_lcg_states", "hpl_ep_set_config", "hpl_ep_launch_shape", "hpl_ep_launch_count",
+)
+
+
+class HPLError(RuntimeError):
+    def __init__(self, code: int, func: str, detail: str):
+        self.code = code
+        super().__init__("%s failed: %s (%d)%s" % (func, _strerror(code), code,
+                                                    (": " + detail) if detail else ""))
+
+
+_lib = None
+
+
+def _load() -> ctypes.CDLL:
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(LIB_PATH):
+        raise ImportError("libhpl.so not built at %s — run `python -m paper_conf_ipps_bozkusf12_b200.build`"
+                          % LIB_PATH)
+    lib = ctypes.CDLL(LIB_PATH)
+    c_int, c_u64, c_i64, c_void_p, c_double = (ctypes.c_int, ctypes.c_uint64, ctypes.c_int64,
+                                              ctypes.c_void_p, ctypes.c_double)
+    P = ctypes.POINTER
+    sig = {
+        "hpl_strerror": (ctypes.c_char_p, [c_int]),
+        "hpl_last_error": (ctypes.c_char_p, []),
+        "hpl_version": (c_int, []),
+        "hpl_device_count": (c_int, [P(c_int)]),
+        "hpl_set_device": (c_int, [c_int]),
+        "hpl_get_device": (c_int, [P(c_int)]),
+        "hpl_array_alloc": (c_int, [P(c_void_p), c_int, c_int, P(c_i64), c_void_p, c_int]),
+        "hpl_array_free": (c_int, [c_void_p]),
+        "hpl_array_sync": (c_int, [c_void_p, c_int, c_int]),
+        "hpl_array_data": (c_int, [c_void_p, c_int, P(c_void_p)]),
+        "hpl_array_info": (c_int, [c_void_p, P(c_int), P(c_int), P(c_i64), P(c_i64), P(c_int)]),
+        "hpl_array_set_stream": (c_int, [c_void_p, c_void_p]),
+        "hpl_ep_eval": (c_int, [c_int, c_u64, c_u64, c_int, c_int, c_void_p]),
+        "hpl_ep_run": (c_int, [c_int, c_u64, c_u64, P(c_double), P(c_double), P(c_u64)]),
+        "hpl_ep_run_shard": (c_int, [c_int, c_u64, c_u64, c_int, c_int, c_void_p, c_void_p]),
+        "hpl_ep_run_range": (c_int, [c_u64, c_u64, c_u64, c_u64, c_void_p, c_void_p]),
+        "hpl_lcg_states": (c_int, [c_u64, c_u64, c_u64, c_u64, P(c_u64)]),
+        "hpl_ep_set_config": (c_int, [c_int, c_int, c_int]),
+        "hpl_ep_launch_shape": (c_int, [c_u64, P(c_int), P(c_int), P(c_int)]),
+        "hpl_ep_launch_count": (c_int, [P(c_u64)]),
+    }
+    for name, (res, args) in sig.items():
+        f = getattr(lib, name)
+        f.restype = res
+        f.argtypes = args
+    _lib = lib
+    return lib
+
+
+def _strerror(code: int) -> str:
+    return _load().hpl_strerror(code).decode()
+
+
+def _check(rc: int, func: str) -> None:
+    if rc != HPL_OK:
+        raise HPLError(rc, func, _load().hpl_last_error().decode())
+
+
+def lib() -> ctypes.CDLL:
+    return _load()
+
+
+# ------------------------------------------------------------------ devices
+def hpl_version() -> int:
+    return _load().hpl_version()
+
+
+def hpl_device_count() -> int:
+    n = ctypes.c_int()
+    _check(_load().hpl_device_count(ctypes.byref(n)), "hpl_device_count")
+    return n.value
+
+
+def hpl_set_device(device: int) -> None:
+    _check(_load().hpl_set_device(device), "hpl_set_device")
+
+
+def hpl_get_device() -> int:
+    d = ctypes.c_int()
+    _check(_load().hpl_get_device(ctypes.byref(d)), "hpl_get_device")
+    return d.value
+
+
+# ------------------------------------------------------------------- arrays
+def hpl_array_alloc(dtype: int, dims, host_ptr=None, device: int = -1) -> int:
+    dims = list(dims)
+    arr = (ctypes.c_int64 * max(len(dims), 1))(*dims)
+    h = ctypes.c_void_p()
+    _check(_load().hpl_array_alloc(ctypes.byref(h), dtype, len(dims), arr, host_ptr, device),
+           "hpl_array_alloc")
+    return h.value
+
+
+def hpl_array_free(a: int) -> None:
+    _check(_load().hpl_array_free(a), "hpl_array_free")
+
+
+def hpl_array_sync(a: int, where: int, mode: int = HPL_READ) -> None:
+    _check(_load().hpl_array_sync(a, where, mode), "hpl_array_sync")
+
+
+def hpl_array_data(a: int, where: int) -> int:
+    p = ctypes.c_void_p()
+    _check(_load().hpl_array_data(a, where, ctypes.byref(p)), "hpl_array_data")
+    return p.value
+
+
+def hpl_array_info(a: int) -> dict:
+    t, nd, nb, v = ctypes.c_int(), ctypes.c_int(), ctypes.c_int64(), ctypes.c_int()
+    dims = (ctypes.c_int64 * 3)()
+    _check(_load().hpl_array_info(a, ctypes.byref(t), ctypes.byref(nd), dims, ctypes.byref(nb),
+                                  ctypes.byref(v)), "hpl_array_info")
+    return {"dtype": t.value, "ndim": nd.value, "dims": list(dims[:nd.value]), "nbytes": nb.value,
+            "valid": v.value}
+
+
+def hpl_array_set_stream(a: int, stream: int | None) -> None:
+    _check(_load().hpl_array_set_stream(a, stream or None), "hpl_array_set_stream")
+
+
+# ----------------------------------------------------------------------- EP
+def hpl_ep_eval(M: int, seed: int, a: int, rank: int, nranks: int, out13: int) -> None:
+    _check(_load().hpl_ep_eval(M, seed, a, rank, nranks, out13), "hpl_ep_eval")
+
+
+def hpl_ep_run(M: int, seed: int, a: int):
+    """Whole EP problem on the current device: returns (sx, sy, q[10])."""
+    sx, sy = ctypes.c_double(), ctypes.c_double()
+    q = (ctypes.c_uint64 * 10)()
+    _check(_load().hpl_ep_run(M, seed, a, ctypes.byref(sx), ctypes.byref(sy), q), "hpl_ep_run")
+    return sx.value, sy.value, list(q)
+
+
+def hpl_ep_run_shard(M: int, seed: int, a: int, rank: int, nranks: int, dev_out13: int,
+                     stream: int | None = None) -> None:
+    _check(_load().hpl_ep_run_shard(M, seed, a, rank, nranks, dev_out13, stream or None),
+           "hpl_ep_run_shard")
+
+
+def hpl_ep_run_range(seed: int, a: int, pair_begin: int, npairs: int, dev_out13: int,
+                     stream: int | None = None) -> None:
+    _check(_load().hpl_ep_run_range(seed, a, pair_begin, npairs, dev_out13, stream or None),
+           "hpl_ep_run_range")
+
+
+def hpl_lcg_states(seed: int, a: int, offset: int, n: int) -> list[int]:
+    buf = (ctypes.c_uint64 * max(n, 1))()
+    _check(_load().hpl_lcg_states(seed, a, offset, n, buf), "hpl_lcg_states")
+    return list(buf[:n])
+
+
+def hpl_ep_set_config(variant: int = HPL_EP_LEAN, threads_per_block: int = 0,
+                      blocks_per_sm: int = 0) -> None:
+    _check(_load().hpl_ep_set_config(variant, threads_per_block, blocks_per_sm), "hpl_ep_set_config")
+
+
+def hpl_ep_launch_shape(npairs: int):
+    b, t, s = ctypes.c_int(), ctypes.c_int(), ctypes.c_int()
+    _check(_load().hpl_ep_launch_shape(npairs, ctypes.byref(b), ctypes.byref(t), ctypes.byref(s)),
+           "hpl_ep_launch_shape")
+    return b.value, t.value, s.value
+
+
+def hpl_ep_launch_count() -> int:
+    c = ctypes.c_uint64()
+    _check(_load().hpl_ep_launch_count(ctypes.byref(c)), "hpl_ep_launch_count")
+    return c.value
+
+
+def unpack13(words) -> dict:
+    """Split the 13-word result [sx, sy, q0..q9, gc] (marshalling helper)."""
+    w = list(words)
+    return {"sx": float(w[0]), "sy": float(w[1]), "q": [int(v) for v in w[2:12]], "gc": int(w[12])}
