@@ -1,0 +1,328 @@
+#!/usr/bin/env python
+"""Benchmark: NPB EP Mops/s (2^(M+1) uniforms / s) on 1..8 B200 (BASELINE.json).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+    torchrun --nproc-per-node N bench.py --gpus N ...        (N > 1, one rank per GPU)
+
+A step = one whole EP problem of class D (M = 36, 2^37 uniforms; the
+BASELINE.json headline config) split over the N ranks: each rank runs its
+shard kernel (hpl_ep_run_shard) and, for N > 1, the 13-word NCCL allreduce.
+EP reads no input arrays (only the (M, seed, a) scalars and a 368-B jump table
+passed as kernel parameters), so "resident in HBM" is vacuous; L2 is flushed
+between timed steps anyway.  Device time: CUDA events per step on the
+launching stream, barrier + synchronize around the timed region, max over
+ranks.  e2e: the same metric through the public API with host results
+(hpl_ep_run / ep_run_distributed incl. the 104-B D2H), wall clock.
+
+--impl reference: the CPU oracle (oracle/, plain NPB EP) on the box's host
+cores over a bounded sample of the same workload — the baseline arm.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from ep_workloads import CLASSES, HEADLINE_CLASS, NPB_A, NPB_SEED, uniforms  # noqa: E402
+
+METRIC = "EP Mops/s (2^(M+1)/s) at 1/2/4/8 B200; fraction of FP64 peak"
+UNIT = "Mops/s"
+PAPER_CONTEXT = {"class": "C", "mops": 3057, "hw": "Tesla C2050/C2070, OpenCL, 2.81 s (PAPER.md:940-942)"}
+
+# Algorithmic FP64 lane-operations per pair: 6 always
+# (2 maps, 2 squares, 1 add, 1 compare) + pi/4 * 19 for accepted pairs
+# (ln 7, sqrt(L/t) 7, X and Y 2, max 1, sums 2).
+ALG_OPS_ALWAYS = 6
+ALG_OPS_ACCEPTED = 19
+P_ACCEPT = 0.7853981633974483
+ALG_OPS_PER_PAIR = ALG_OPS_ALWAYS + P_ACCEPT * ALG_OPS_ACCEPTED
+FP64_LANES_PER_SM_CLK = 64          # measured: tools/probe_fp64.cu (63.9-64.1 lane-DFMA/clk/SM)
+EP_PARAM_BYTES = 440                 # EPParams kernel-parameter block (jump table + scalars)
+
+
+def peaks():
+    p = {}
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(path):
+        p = json.load(open(path))
+    return p
+
+
+def load_profile_traffic():
+    """dram bytes per launch of the EP kernel from the committed ncu summary, or None."""
+    path = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    if not os.path.exists(path):
+        return None
+    try:
+        return json.load(open(path)).get("dram_bytes_per_launch")
+    except Exception:
+        return None
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.sw_power_cap,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.rows = []
+        self.proc = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), "--query-gpu=" + self.FIELDS,
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.thread = threading.Thread(target=self._read, daemon=True)
+            self.thread.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) == 7:
+                self.rows.append(parts)
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        rows = self.rows
+        names = ["sw_power_cap", "hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown"]
+        sm = [float(r[0]) for r in rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
+        pw = [float(r[2]) for r in rows if r[2].replace(".", "").isdigit()]
+        active = sorted({names[i] for r in rows for i in range(4) if r[3 + i].lower().startswith("active")})
+        loaded = [s for s in sm if mx and s > 0.5 * max(mx)] or sm
+        return {"sm_mhz": statistics.median(loaded) if loaded else None,
+                "sm_max_mhz": max(mx) if mx else None,
+                "power_w_max": max(pw) if pw else None,
+                "samples": len(rows), "reasons": active}
+
+
+# --------------------------------------------------------------- reference
+def run_reference(args, M):
+    import oracle
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    threads = os.cpu_count() or 1
+    nb_total = 1 << (M - 16)
+    # bounded sample: `batches` NPB batches (2^16 pairs each) per step
+    batches = min(nb_total, args.ref_batches or 64 * threads)
+    for _ in range(args.warmup):
+        oracle.run_batches(M, NPB_SEED, NPB_A, 0, min(batches, threads), threads=threads, margin=False)
+    ts = []
+    for s in range(args.steps):
+        k0 = (s * batches) % max(nb_total - batches + 1, 1)
+        t0 = time.perf_counter()
+        oracle.run_batches(M, NPB_SEED, NPB_A, k0, k0 + batches, threads=threads, margin=False)
+        ts.append(time.perf_counter() - t0)
+    pairs = batches << 16
+    tot = sum(ts)
+    value = 2 * pairs * args.steps / tot / 1e6
+    sample = ("NPB batches [k0, k0+%d) of class %s (2^16 pairs each, %d uniforms per step), "
+              "batch-parallel over %d threads, margin tracking off" % (batches, args.cls, 2 * pairs, threads))
+    line = {
+        "impl": "reference", "metric": METRIC, "value": round(value, 3), "unit": UNIT,
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round(tot / args.steps * 1e3, 3), "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic (NPB LCG stream)",
+        "config": {"workload": "NPB EP class %s (M=%d)" % (args.cls, M), "M": M, "seed": NPB_SEED,
+                   "a": NPB_A, "sampled": True},
+        "cpu_baseline": {"value": round(value, 3), "unit": UNIT, "cores": threads, "kind": "oracle",
+                         "sample": sample},
+        "e2e": {"value": round(value, 3), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def cpu_baseline_sample(M, budget_s):
+    """Oracle as it stands on the host cores over a bounded sample of class M."""
+    import oracle
+    threads = os.cpu_count() or 1
+    t0 = time.perf_counter()
+    oracle.run_batches(M, NPB_SEED, NPB_A, 0, threads, threads=threads, margin=False)
+    t_one = max(time.perf_counter() - t0, 1e-3)  # one batch per thread
+    batches = max(threads, int(budget_s / t_one) * threads)
+    batches = min(batches, 1 << (M - 16))
+    t0 = time.perf_counter()
+    oracle.run_batches(M, NPB_SEED, NPB_A, 0, batches, threads=threads, margin=False)
+    dt = time.perf_counter() - t0
+    pairs = batches << 16
+    return {"value": round(2 * pairs / dt / 1e6, 3), "unit": UNIT, "cores": threads, "kind": "oracle",
+            "sample": "first %d NPB batches of class-%d stream (%d pairs, %.1f s), batch-parallel over "
+                      "%d threads, margin tracking off" % (batches, M, pairs, dt, threads)}
+
+
+# --------------------------------------------------------------------- ours
+def run_ours(args, M):
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_ipps_bozkusf12_b200 import hpl, multi
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        raise SystemExit("--gpus %d but WORLD_SIZE=%d (launch with torchrun for N>1)" % (args.gpus, world))
+    torch.cuda.set_device(local)
+    hpl.hpl_set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    stream = torch.cuda.current_stream(dev)
+    out = torch.empty(13, dtype=torch.float64, device=dev)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # > 126 MB L2
+
+    def step():
+        hpl.hpl_ep_run_shard(M, NPB_SEED, NPB_A, rank, world, out.data_ptr(), stream.cuda_stream)
+
+    for _ in range(args.warmup):
+        step()
+        if world > 1:
+            dist.all_reduce(out)
+    torch.cuda.synchronize(dev)
+
+    # ---- device-timed region
+    sampler = ClockSampler(local)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize(dev)
+    sampler.start()
+    launches0 = hpl.hpl_ep_launch_count()
+    step_ms, kern_ms = [], []
+    for _ in range(args.steps):
+        flush.zero_()  # untimed L2 flush between steps
+        e0, e1, e2 = (torch.cuda.Event(enable_timing=True) for _ in range(3))
+        e0.record(stream)
+        step()
+        e1.record(stream)
+        if world > 1:
+            dist.all_reduce(out)
+        e2.record(stream)
+        e2.synchronize()
+        kern_ms.append(e0.elapsed_time(e1))
+        step_ms.append(e0.elapsed_time(e2))
+    torch.cuda.synchronize(dev)
+    launches = hpl.hpl_ep_launch_count() - launches0
+    if world > 1:
+        dist.barrier()
+    clocks = sampler.stop()
+    result = hpl.unpack13(out.cpu().tolist())
+
+    total_ms = sum(step_ms)
+    t = torch.tensor([total_ms, sum(kern_ms), float(launches)], dtype=torch.float64, device=dev)
+    if world > 1:
+        tmax = t.clone()
+        dist.all_reduce(tmax, op=dist.ReduceOp.MAX)
+        tsum = t.clone()
+        dist.all_reduce(tsum, op=dist.ReduceOp.SUM)
+        total_ms, kern_max_ms, launches_all = tmax[0].item(), tmax[1].item(), int(tsum[2].item())
+    else:
+        kern_max_ms, launches_all = sum(kern_ms), launches
+
+    # ---- e2e through the public API (host results)
+    e2e_ms = []
+    if world > 1:
+        dist.barrier()
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        if world == 1:
+            sx, sy, q = hpl.hpl_ep_run(M, NPB_SEED, NPB_A)  # blocking, 104-B D2H inside
+        else:
+            multi.ep_run_distributed(M, NPB_SEED, NPB_A, device=dev)
+        e2e_ms.append((time.perf_counter() - t0) * 1e3)
+    e2e_tot = sum(e2e_ms)
+    if world > 1:
+        te = torch.tensor([e2e_tot], dtype=torch.float64, device=dev)
+        dist.all_reduce(te, op=dist.ReduceOp.MAX)
+        e2e_tot = te.item()
+
+    if rank == 0:
+        units = uniforms(M)
+        value = units * args.steps / (total_ms / 1e3) / 1e6
+        # roofline of the dominant (only) kernel: algorithmic FP64 lane-ops per launch
+        pk = peaks()
+        sm_max = float(pk.get("sm_max_mhz", 1965.0))
+        props = torch.cuda.get_device_properties(dev)
+        peak_ops = props.multi_processor_count * FP64_LANES_PER_SM_CLK * sm_max * 1e6
+        pairs_per_launch = (1 << M) // world
+        kern_avg_s = kern_max_ms / args.steps / 1e3
+        achieved = ALG_OPS_PER_PAIR * pairs_per_launch / kern_avg_s
+        traffic = load_profile_traffic()
+        line = {
+            "metric": METRIC, "value": round(value, 1), "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": round(total_ms / args.steps, 4), "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic (NPB LCG stream, seed 271828183, a=5^13)",
+            "config": {"workload": "NPB EP class %s (M=%d)" % (args.cls, M), "M": M,
+                       "global_pairs": 1 << M, "seed": NPB_SEED, "a": NPB_A,
+                       "parallelism": "shard x%d + allreduce(13 x f64)" % world if world > 1 else "1 GPU",
+                       "l2": "flushed (256 MB write) between timed steps; EP reads no inputs",
+                       "kernel_shape": list(hpl.hpl_ep_launch_shape(pairs_per_launch))},
+            "paper_context": PAPER_CONTEXT,
+            "roofline": {"bound": "alu", "achieved": round(achieved / 1e12, 3),
+                         "peak": round(peak_ops / 1e12, 3), "unit": "FP64 Tops/s (lane-ops)",
+                         "frac": round(achieved / peak_ops, 4), "traffic": traffic,
+                         "alg_ops_per_pair": round(ALG_OPS_PER_PAIR, 3),
+                         "peak_basis": "%d SMs x %d FP64 lanes/clk x %.0f MHz (sm_max_mhz)"
+                                       % (props.multi_processor_count, FP64_LANES_PER_SM_CLK, sm_max),
+                         "kernel_ms": round(kern_avg_s * 1e3, 4)},
+            "e2e": {"value": round(units * args.steps / (e2e_tot / 1e3) / 1e6, 1), "unit": UNIT,
+                    "h2d_bytes_per_step": EP_PARAM_BYTES * world, "d2h_bytes_per_step": 104 * world,
+                    "note": "h2d = kernel-parameter block (jump table + scalars); d2h = 13-word result"},
+            "gpu_launches": launches_all,
+            "clocks": clocks,
+            "result": {"sx": result["sx"], "sy": result["sy"], "gc": result["gc"]},
+        }
+        if not args.no_cpu_baseline and world == 1:
+            line["cpu_baseline"] = cpu_baseline_sample(M, args.cpu_budget)
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser(description=__doc__, formatter_class=argparse.RawDescriptionHelpFormatter)
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--cls", default=HEADLINE_CLASS, choices=sorted(CLASSES))
+    ap.add_argument("--cpu-budget", type=float, default=15.0, help="seconds of oracle work for cpu_baseline")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--ref-batches", type=int, default=0, help="NPB batches per --impl reference step")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        ap.error("--warmup must be >= 3")
+    M = CLASSES[args.cls]
+    if args.impl == "reference":
+        return run_reference(args, M)
+    return run_ours(args, M)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

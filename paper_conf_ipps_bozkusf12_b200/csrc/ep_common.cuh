@@ -35,21 +35,27 @@ EP_HD uint64_t step_v(uint64_t v, uint64_t a) { return ((a * v) & MASK52) | EXP_
 constexpr int NJUMP = 46;
 
 // ---- lean-log table ---------------------------------------
-// -2 ln t for t in (0, 1] is computed as T[u] + r * q(r) where
-// u indexes (exponent, top LOG_K mantissa bits) of t rounded to the nearest
-// bucket centre, inv[u] is a float-exact approximation of 1/centre,
-// r = fma(t, inv[u], -1) and T[u] = RN(2 ln inv[u]).
+// The kernel works with t' = t/4 in (0, 1/4] (x' = x/2, exact).  -2 ln t is
+// computed as T[u] + r * q(r) where u indexes (exponent, top LOG_K mantissa
+// bits) of t' rounded to the nearest bucket centre c, inv[u] is a
+// float-exact approximation of 1/c, r = fma(t', inv[u], -1) (|r| <= 2^-9) and
+// T[u] = RN(2 ln(inv[u] / 4)), so that -2 ln t = T[u] - 2 ln(1 + r).
 constexpr int LOG_K = 8;                       // mantissa bits per exponent
-constexpr int LOG_EMIN = -16;                  // smallest exponent in the table
+constexpr int LOG_EMIN = -16;                  // table covers t >= ~2^LOG_EMIN
 constexpr int LOG_SHIFT = 20 - LOG_K;          // hi-word shift to the index
-constexpr uint32_t LOG_IDX_MIN = uint32_t(1023 + LOG_EMIN) << LOG_K;
-constexpr uint32_t LOG_IDX_MAX = uint32_t(1023) << LOG_K;  // bucket of t = 1.0
-constexpr uint32_t LOG_N = LOG_IDX_MAX - LOG_IDX_MIN + 1;  // 4097 entries
-// u = (hi(t) + LOG_ADD) >> LOG_SHIFT  (mod 2^32), valid iff u < LOG_N
+constexpr uint32_t LOG_BIAS_TOP = 1023 - 2;    // biased exponent of t' = 1/4
+constexpr uint32_t LOG_IDX_MIN = uint32_t(LOG_BIAS_TOP + LOG_EMIN) << LOG_K;
+constexpr uint32_t LOG_IDX_MAX = uint32_t(LOG_BIAS_TOP) << LOG_K;  // bucket of t' = 1/4
+constexpr uint32_t LOG_N = LOG_IDX_MAX - LOG_IDX_MIN + 1;  // 4097 real entries
+// u = (hi(t') + LOG_ADD) >> LOG_SHIFT  (mod 2^32), valid iff u < LOG_N
 constexpr uint32_t LOG_ADD = (uint32_t(1) << (LOG_SHIFT - 1)) - (LOG_IDX_MIN << LOG_SHIFT);
+// Entry LOG_N is a sentinel {T = 2^1000, inv = 0}: every t' outside the table
+// (rejected t' > ~1/4, or t < 2^LOG_EMIN) is clamped onto it, which makes
+// t2 ~ 2^500 and hence l >= 4, routing the pair to the exact rare path.
+constexpr uint32_t LOG_TAB = LOG_N + 1;
 
 struct LogEntry {
-  double T;    // RN(2 ln inv)
+  double T;    // RN(2 ln(inv / 4))
   double inv;  // float-representable ~1/centre
 };
 
@@ -62,12 +68,14 @@ struct EPPartial {
 
 struct EPParams {
   uint64_t jump[NJUMP];  // a^(2^i) mod 2^46
+  double coef[6];        // lean constants (kept in the parameter bank, not registers)
   uint64_t a;            // multiplier
+  unsigned a_lo, a_hi;   // its 32-bit halves
   uint64_t x_begin;      // state before the first uniform of this launch's range
   uint64_t npairs;       // pairs in this launch
   uint64_t base;         // pairs per thread (floor)
   uint64_t extra;        // threads [0, extra) take base + 1 pairs
-  const LogEntry* table; // global copy of the lean-log table (LOG_N entries)
+  const LogEntry* table; // global copy of the lean-log table (LOG_TAB entries)
   EPPartial* partials;   // [gridDim.x]
   unsigned int* counter; // last-block-done ticket, left at 0 after each launch
   double* out13;         // result

@@ -45,17 +45,136 @@ __device__ __forceinline__ double rsqrt_approx(double p) {
   return y;
 }
 
-__device__ __forceinline__ unsigned shl_clamped(unsigned x, unsigned s) {
+// 1 << (8 l) for l in 0..3 in one PRMT (backward-4-extract of the byte string
+// {1,0,0,0,0,0,0,0} starting at byte l); lanes with l >= 4 never use it.
+__device__ __forceinline__ unsigned bin_increment(unsigned l) {
   unsigned r;
-  asm("shl.b32 %0, %1, %2;" : "=r"(r) : "r"(x), "r"(s));  // s >= 32 -> 0 (PTX clamps)
+  asm("prmt.b32.b4e %0, %1, %2, %3;" : "=r"(r) : "r"(1u), "r"(0u), "r"(l));
   return r;
 }
 
-template <int VARIANT, bool A32>
-__global__ void __launch_bounds__(EP_MAX_THREADS)
+// One LCG step on the (lo, hi) words of v = bits(1 + x 2^-46):
+//   v' = ((a v) mod 2^52) | bits(1.0)
+// = IMAD.WIDE.U32 + IMAD (+ IMAD if a >= 2^32) + one LOP3 doing mask and OR.
+template <bool A32>
+__device__ __forceinline__ void lcg_step(unsigned& lo, unsigned& hi, unsigned a_lo, unsigned a_hi) {
+  const unsigned ph = __umulhi(lo, a_lo) + hi * a_lo + (A32 ? 0u : lo * a_hi);
+  lo = lo * a_lo;
+  hi = (ph & 0x000FFFFFu) | 0x3FF00000u;
+}
+
+
+struct PairAcc {
+  double csx, csy;
+  unsigned cnt;  // 8-bit packed counts of bins 0..3
+};
+
+// Exact slow path for the rare lanes: t below the table (sentinel) or
+// l >= 4.  Recomputes what the fast path could not and tallies bins >= 4 in
+// shared memory; returns the sums/count increments (registers, no locals).
+struct RareOut {
+  double dx, dy;
+  unsigned dcnt;
+};
+__device__ __noinline__ RareOut rare_pair(double t, double x1, double x2, double X, double Y,
+                                          unsigned u, unsigned long long* s_rare) {
+  if (u >= LOG_N) {  // t below the table: NPB's formula, libdevice log/sqrt, on
+    // the unscaled t = 4 t', x = 2 x' (exact)
+    const double tt = 4.0 * t;
+    const double t2 = sqrt(-2.0 * log(tt) / tt);
+    X = __dmul_rn(2.0 * x1, t2);
+    Y = __dmul_rn(2.0 * x2, t2);
+  }
+  const unsigned l = __double2uint_rz(fmax(fabs(X), fabs(Y)));
+  RareOut o{X, Y, 0u};
+  if (l < 4) o.dcnt = bin_increment(l);
+  else atomicAdd(&s_rare[(l < 10 ? l : 10u) - 4], 1ull);
+  return o;
+}
+
+// One pair, lean transform (A3-A7).  No branch on the common path: rejected
+// lanes compute garbage that the `ok` predicate discards.
+//
+// Scaled variables (exact, powers of two): x' = v - 1.5 = x/2, t' = x1'^2 +
+// x2'^2 = t/4 (same roundings as NPB's t), accept iff t' <= 1/4.  The table is
+// indexed by t' and returns L = -2 ln t directly; t2' = sqrt(L/t') = 2 t2, so
+// X = x1' t2' = x1 t2 exactly as NPB's X.
+template <bool A32>
+__device__ __forceinline__ void lean_pair(unsigned& vlo, unsigned& vhi, const EPParams& P,
+                                          unsigned tab, PairAcc& A, unsigned long long* s_rare) {
+  lcg_step<A32>(vlo, vhi, P.a_lo, P.a_hi);
+  const double v1 = __hiloint2double(int(vhi), int(vlo));
+  lcg_step<A32>(vlo, vhi, P.a_lo, P.a_hi);
+  const double v2 = __hiloint2double(int(vhi), int(vlo));
+  const double x1 = __dadd_rn(v1, -1.5);  // (2u - 1)/2, exact
+  const double x2 = __dadd_rn(v2, -1.5);
+  const double t = __dadd_rn(__dmul_rn(x1, x1), __dmul_rn(x2, x2));  // t/4, NPB roundings (R5)
+  const bool acc = t <= 0.25;
+  // A5: L = -2 ln(4 t) from the table entry of t (sentinel for t outside)
+  const unsigned H = static_cast<unsigned>(__double2hiint(t));
+  const unsigned u = min((H + LOG_ADD) >> LOG_SHIFT, LOG_N);
+  double eT, eInv;
+  asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(eT), "=d"(eInv) : "r"(tab + u * 16u));
+  const double r = fma(t, eInv, -1.0);
+  double c = fma(P.coef[0], r, P.coef[1]);
+  c = fma(c, r, 0.5);
+  c = fma(c, r, P.coef[2]);
+  c = fma(c, r, 1.0);
+  c = fma(c, r, -2.0);
+  const double L = fma(c, r, eT);
+  // t2' = sqrt(L/t) = L rsqrt(L t): MUFU seed + one cubic Newton step
+  const double p = fma(L, t, P.coef[5]);  // + 2^-200: t' == 1/4 -> L = 0 -> t2' = 0
+  const double y0 = rsqrt_approx(p);
+  const double h = __dmul_rn(p, y0);
+  const double e = fma(-h, y0, 1.0);
+  const double cc = fma(e, P.coef[3], 0.5);
+  const double g = __dmul_rn(L, y0);
+  const double ge = __dmul_rn(g, e);
+  const double t2 = fma(ge, cc, g);
+  // A6/A7 as NPB writes them: X = x1 t2, Y = x2 t2, l = int(max(|X|,|Y|))
+  const double X = __dmul_rn(x1, t2);
+  const double Y = __dmul_rn(x2, t2);
+  const unsigned l = max(__double2uint_rz(fabs(X)), __double2uint_rz(fabs(Y)));
+  const bool ok = acc && l < 4;
+  if (ok) {
+    A.csx = __dadd_rn(A.csx, X);
+    A.csy = __dadd_rn(A.csy, Y);
+    A.cnt += bin_increment(l);
+  }
+  if (acc && !ok) {
+    const RareOut o = rare_pair(t, x1, x2, X, Y, u, s_rare);
+    A.csx += o.dx;
+    A.csy += o.dy;
+    A.cnt += o.dcnt;
+  }
+}
+
+// NPB's own formulation with CUDA libdevice log / div / sqrt (A/B variant).
+template <bool A32>
+__device__ __forceinline__ void libdevice_pair(unsigned& vlo, unsigned& vhi, const EPParams& P,
+                                               unsigned, PairAcc& A, unsigned long long* s_rare) {
+  lcg_step<A32>(vlo, vhi, P.a_lo, P.a_hi);
+  const double v1 = __hiloint2double(int(vhi), int(vlo));
+  lcg_step<A32>(vlo, vhi, P.a_lo, P.a_hi);
+  const double v2 = __hiloint2double(int(vhi), int(vlo));
+  const double x1 = fma(v1, 2.0, -3.0);
+  const double x2 = fma(v2, 2.0, -3.0);
+  const double t = __dadd_rn(__dmul_rn(x1, x1), __dmul_rn(x2, x2));
+  if (t <= 1.0) {
+    const double t2 = sqrt(-2.0 * log(t) / t);
+    const double X = __dmul_rn(x1, t2), Y = __dmul_rn(x2, t2);
+    const unsigned l = __double2uint_rz(fmax(fabs(X), fabs(Y)));
+    A.csx += X;
+    A.csy += Y;
+    if (l < 4) A.cnt += bin_increment(l);
+    else atomicAdd(&s_rare[(l < 10 ? l : 10u) - 4], 1ull);
+  }
+}
+
+template <int VARIANT, bool A32, int NT, int MINB>
+__global__ void __launch_bounds__(NT, MINB)
 ep_kernel(const __grid_constant__ EPParams P) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
-  LogEntry* s_tab = reinterpret_cast<LogEntry*>(smem_raw);
   __shared__ unsigned long long s_rare[7];  // bins 4..9, then l >= 10
   __shared__ double s_wsx[EP_MAX_THREADS / 32], s_wsy[EP_MAX_THREADS / 32];
   __shared__ unsigned long long s_wq[EP_MAX_THREADS / 32][4];
@@ -63,10 +182,11 @@ ep_kernel(const __grid_constant__ EPParams P) {
   __shared__ double s_fin[13];
 
   const unsigned tid = threadIdx.x;
+  const unsigned tab = static_cast<unsigned>(__cvta_generic_to_shared(smem_raw));
   if (VARIANT == HPL_VARIANT_LEAN) {
     const double2* src = reinterpret_cast<const double2*>(P.table);
-    double2* dst = reinterpret_cast<double2*>(s_tab);
-    for (unsigned i = tid; i < LOG_N; i += blockDim.x) dst[i] = __ldg(src + i);
+    double2* dst = reinterpret_cast<double2*>(smem_raw);
+    for (unsigned i = tid; i < LOG_TAB; i += blockDim.x) dst[i] = __ldg(src + i);
   }
   if (tid < 7) s_rare[tid] = 0;
   __syncthreads();
@@ -75,82 +195,42 @@ ep_kernel(const __grid_constant__ EPParams P) {
   const uint64_t gid = uint64_t(blockIdx.x) * blockDim.x + tid;
   const uint64_t n_t = P.base + (gid < P.extra ? 1 : 0);
   const uint64_t p0 = gid * P.base + (gid < P.extra ? gid : P.extra);
-  uint64_t v = state_to_v(jump_state(P.x_begin, 2 * p0, P.jump));
-  const uint64_t a = A32 ? (P.a & 0xFFFFFFFFull) : P.a;
+  const uint64_t v0 = state_to_v(jump_state(P.x_begin, 2 * p0, P.jump));
+  unsigned vlo = unsigned(v0), vhi = unsigned(v0 >> 32);
 
   double sx = 0.0, sy = 0.0;
   unsigned q0 = 0, q1 = 0, q2 = 0, q3 = 0;
+  auto flush = [&](const PairAcc& A) {
+    q0 += A.cnt & 0xFFu;
+    q1 += (A.cnt >> 8) & 0xFFu;
+    q2 += (A.cnt >> 16) & 0xFFu;
+    q3 += A.cnt >> 24;
+    sx += A.csx;
+    sy += A.csy;
+  };
+  // 8-bit packed counters overflow after 255 pairs: chunks of 252 = 63 x 4
+  constexpr unsigned UNROLL = 4, CHUNK = 63 * UNROLL;
   uint64_t rem = n_t;
-  while (rem != 0) {
-    // 8-bit packed counters for bins 0..3 overflow after 255 pairs
-    const unsigned chunk = rem < 255 ? unsigned(rem) : 255u;
-    unsigned cnt = 0;
-    double csx = 0.0, csy = 0.0;
-#pragma unroll 4
-    for (unsigned i = 0; i < chunk; ++i) {
-      // ---- A3: two LCG steps; v is the bit pattern of 1 + u
-      v = step_v(v, a);
-      const double v1 = as_double(v);
-      v = step_v(v, a);
-      const double v2 = as_double(v);
-      // ---- A4: x = 2u - 1 = 2v - 3 (exact); t unfused like NPB (R5)
-      const double x1 = fma(v1, 2.0, -3.0);
-      const double x2 = fma(v2, 2.0, -3.0);
-      const double t = __dadd_rn(__dmul_rn(x1, x1), __dmul_rn(x2, x2));
-      const bool acc = t <= 1.0;
-      if (VARIANT == HPL_VARIANT_LIBDEVICE) {
-        // NPB's own formulation: t2 = sqrt(-2 log t / t), X = x1 t2, Y = x2 t2
-        if (acc) {
-          const double t2 = sqrt(-2.0 * log(t) / t);
-          const double X = __dmul_rn(x1, t2), Y = __dmul_rn(x2, t2);
-          const unsigned l = __double2uint_rz(fmax(fabs(X), fabs(Y)));
-          csx += X;
-          csy += Y;
-          cnt += shl_clamped(1u, l << 3);
-          if (l >= 4) atomicAdd(&s_rare[(l < 10 ? l : 10u) - 4], 1ull);
-        }
-      } else {
-        // ---- A5 lean: L = -2 ln t = T[u] + r q(r) (table + degree-6 series)
-        const unsigned H = static_cast<unsigned>(__double2hiint(t));
-        const unsigned u = (H + LOG_ADD) >> LOG_SHIFT;
-        const unsigned uc = u < LOG_N ? u : LOG_N - 1;
-        const double2 ent = reinterpret_cast<const double2*>(s_tab)[uc];
-        const double r = fma(t, ent.y, -1.0);
-        double c = fma(1.0 / 3.0, r, -0.4);
-        c = fma(c, r, 0.5);
-        c = fma(c, r, -2.0 / 3.0);
-        c = fma(c, r, 1.0);
-        c = fma(c, r, -2.0);
-        double L = fma(c, r, ent.x);
-        if (acc && u >= LOG_N) L = -2.0 * log(t);  // t < 2^-16: rare slow path
-        // t2 = sqrt(L / t) = L * rsqrt(L t); one cubic Newton step from MUFU
-        const double p = fma(L, t, 0x1p-200);  // + tiny: t == 1 gives L = 0 -> t2 = 0
-        const double y0 = rsqrt_approx(p);
-        const double h = __dmul_rn(p, y0);
-        const double e = fma(-h, y0, 1.0);
-        const double cc = fma(e, 0.375, 0.5);
-        const double g = __dmul_rn(L, y0);
-        const double ge = __dmul_rn(g, e);
-        const double t2 = fma(ge, cc, g);
-        // ---- A6: l = trunc(RN(max(|x1|,|x2|) t2)) == trunc(max(|X|,|Y|))
-        const double mm = __dmul_rn(fmax(fabs(x1), fabs(x2)), t2);
-        const unsigned l = __double2uint_rz(mm);
-        if (acc) {
-          // ---- A7
-          csx = fma(x1, t2, csx);
-          csy = fma(x2, t2, csy);
-          cnt += shl_clamped(1u, l << 3);
-          if (l >= 4) atomicAdd(&s_rare[(l < 10 ? l : 10u) - 4], 1ull);
-        }
+  for (; rem >= CHUNK; rem -= CHUNK) {
+    PairAcc A{0.0, 0.0, 0u};
+#pragma unroll 1
+    for (unsigned i = 0; i < CHUNK / UNROLL; ++i) {
+#pragma unroll
+      for (unsigned j = 0; j < UNROLL; ++j) {
+        if (VARIANT == HPL_VARIANT_LEAN) lean_pair<A32>(vlo, vhi, P, tab, A, s_rare);
+        else libdevice_pair<A32>(vlo, vhi, P, tab, A, s_rare);
       }
     }
-    q0 += cnt & 0xFFu;
-    q1 += (cnt >> 8) & 0xFFu;
-    q2 += (cnt >> 16) & 0xFFu;
-    q3 += cnt >> 24;
-    sx += csx;
-    sy += csy;
-    rem -= chunk;
+    flush(A);
+  }
+  if (rem) {
+    PairAcc A{0.0, 0.0, 0u};
+#pragma unroll 1
+    for (unsigned i = 0; i < unsigned(rem); ++i) {
+      if (VARIANT == HPL_VARIANT_LEAN) lean_pair<A32>(vlo, vhi, P, tab, A, s_rare);
+      else libdevice_pair<A32>(vlo, vhi, P, tab, A, s_rare);
+    }
+    flush(A);
   }
 
   // ---- A8: warp -> block reduction (fixed order => deterministic)
@@ -232,6 +312,23 @@ __global__ void lcg_states_kernel(uint64_t seed, uint64_t a, uint64_t offset, ui
   out[i] = v_to_state(v);
 }
 
+// ------------------------------------------------------------- dispatcher
+// Launch-bound tiers: (max threads per block, min blocks per SM) -> register cap
+// 64 / 64 / 85 / 85 / 128 regs.  A launch uses the smallest tier >= its block.
+using EPKernel = void (*)(const EPParams);
+template <int V, bool A32>
+static EPKernel tier_kernel(int thr) {
+  if (thr <= 128) return ep_kernel<V, A32, 128, 4>;
+  if (thr <= 256) return ep_kernel<V, A32, 256, 3>;
+  if (thr <= 384) return ep_kernel<V, A32, 384, 2>;
+  if (thr <= 512) return ep_kernel<V, A32, 512, 2>;
+  return ep_kernel<V, A32, 1024, 1>;
+}
+static EPKernel pick_kernel(int variant, bool a32, int thr) {
+  if (variant == HPL_VARIANT_LEAN) return a32 ? tier_kernel<HPL_VARIANT_LEAN, true>(thr) : tier_kernel<HPL_VARIANT_LEAN, false>(thr);
+  return a32 ? tier_kernel<HPL_VARIANT_LIBDEVICE, true>(thr) : tier_kernel<HPL_VARIANT_LIBDEVICE, false>(thr);
+}
+
 // ------------------------------------------------------------------ host side
 void build_jump_table(uint64_t a, uint64_t* J) {
   uint64_t x = a & MASK46;
@@ -249,15 +346,17 @@ uint64_t host_jump(uint64_t x, uint64_t k, const uint64_t* J) {
 
 // Lean-log table, built in 80-bit long double on the host.
 void build_log_table(std::vector<LogEntry>& tab) {
-  tab.resize(LOG_N);
+  tab.resize(LOG_TAB);
   for (uint32_t u = 0; u < LOG_N; ++u) {
     const uint32_t idx = LOG_IDX_MIN + u;
     const int E = int(idx >> LOG_K) - 1023;
     const long double centre = ldexpl(1.0L + (long double)(idx & ((1u << LOG_K) - 1)) / (1 << LOG_K), E);
     const float inv = (float)(1.0L / centre);
     tab[u].inv = (double)inv;
-    tab[u].T = (double)(2.0L * logl((long double)inv));
+    tab[u].T = (double)(2.0L * logl((long double)inv * 0.25L));  // -2 ln(4 t') at r = 0
   }
+  tab[LOG_N].T = 0x1p1000;  // sentinel: forces l >= 4 -> exact rare path
+  tab[LOG_N].inv = 0.0;
 }
 
 namespace {
@@ -282,12 +381,13 @@ int set_attrs_once(int device) {
   static std::vector<char> done;
   if ((int)done.size() <= device) done.resize(device + 1, 0);
   if (done[device]) return 0;
-  const int smem = int(LOG_N * sizeof(LogEntry));
-  cudaError_t e;
-  e = cudaFuncSetAttribute(ep_kernel<HPL_VARIANT_LEAN, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  if (e == cudaSuccess)
-    e = cudaFuncSetAttribute(ep_kernel<HPL_VARIANT_LEAN, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  if (e != cudaSuccess) return set_cuda_error(e, "cudaFuncSetAttribute");
+  const int smem = int(LOG_TAB * sizeof(LogEntry));
+  for (int thr : {128, 256, 384, 512, 1024})
+    for (bool a32 : {true, false}) {
+      cudaError_t e = cudaFuncSetAttribute(pick_kernel(HPL_VARIANT_LEAN, a32, thr),
+                                           cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+      if (e != cudaSuccess) return set_cuda_error(e, "cudaFuncSetAttribute");
+    }
   done[device] = 1;
   return 0;
 }
@@ -357,13 +457,12 @@ int launch_shape(int device, uint64_t npairs, const EPConfig& cfg, int* blocks, 
   if (rc) return rc;
   const int thr = cfg.threads_per_block > 0 ? cfg.threads_per_block : EP_DEFAULT_THREADS;
   if (thr < 32 || thr > EP_MAX_THREADS || thr % 32) return set_error(HPL_EINVAL, "threads_per_block must be a multiple of 32 in [32, 1024]");
-  const int sm_bytes = cfg.variant == HPL_VARIANT_LEAN ? int(LOG_N * sizeof(LogEntry)) : 0;
+  const int sm_bytes = cfg.variant == HPL_VARIANT_LEAN ? int(LOG_TAB * sizeof(LogEntry)) : 0;
   int bps = cfg.blocks_per_sm;
   if (bps <= 0) {
     int occ = 0;
-    cudaError_t e = cfg.variant == HPL_VARIANT_LEAN
-        ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ep_kernel<HPL_VARIANT_LEAN, true>, thr, sm_bytes)
-        : cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ep_kernel<HPL_VARIANT_LIBDEVICE, true>, thr, 0);
+    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, pick_kernel(cfg.variant, true, thr),
+                                                                  thr, sm_bytes);
     if (e != cudaSuccess) return set_cuda_error(e, "cudaOccupancyMaxActiveBlocksPerMultiprocessor");
     bps = occ > 0 ? occ : 1;
   }
@@ -396,6 +495,10 @@ int launch_ep(int device, uint64_t seed, uint64_t a, uint64_t pair_begin, uint64
   std::memset(&P, 0, sizeof(P));
   build_jump_table(a, P.jump);
   P.a = a;
+  P.a_lo = unsigned(a);
+  P.a_hi = unsigned(a >> 32);
+  const double coef[6] = {1.0 / 3.0, -0.4, -2.0 / 3.0, 0.375, 0.5, 0x1p-200};
+  for (int i = 0; i < 6; ++i) P.coef[i] = coef[i];
   P.x_begin = host_jump(seed & MASK46, 2 * pair_begin, P.jump);
   P.npairs = npairs;
   const uint64_t T = uint64_t(blocks) * threads;
@@ -407,13 +510,7 @@ int launch_ep(int device, uint64_t seed, uint64_t a, uint64_t pair_begin, uint64
   P.out13 = dev_out13;
 
   const bool a32 = (a >> 32) == 0;
-  if (cfg.variant == HPL_VARIANT_LEAN) {
-    if (a32) ep_kernel<HPL_VARIANT_LEAN, true><<<blocks, threads, smem, stream>>>(P);
-    else ep_kernel<HPL_VARIANT_LEAN, false><<<blocks, threads, smem, stream>>>(P);
-  } else {
-    if (a32) ep_kernel<HPL_VARIANT_LIBDEVICE, true><<<blocks, threads, 0, stream>>>(P);
-    else ep_kernel<HPL_VARIANT_LIBDEVICE, false><<<blocks, threads, 0, stream>>>(P);
-  }
+  pick_kernel(cfg.variant, a32, threads)<<<blocks, threads, smem, stream>>>(P);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return set_cuda_error(e, "ep_kernel launch");
   {

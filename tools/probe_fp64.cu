@@ -48,6 +48,45 @@ __global__ void rsqrt_err(const double* x, double* rel_rs, double* rel_rc, int n
   rel_rc[i] = fabs(z - 1.0 / v) * v;
 }
 
+
+// Dependent-chain latencies (one warp): cycles per dependent instruction.
+__global__ void lat_kernel(double* out, long long* cyc, double x, int n) {
+  __shared__ double2 sm[256];
+  for (int i = threadIdx.x; i < 256; i += blockDim.x) sm[i] = make_double2(1.0 + i * 1e-3, 0.5);
+  __syncthreads();
+  double a = x + threadIdx.x * 1e-9, b = a;
+  unsigned u = threadIdx.x;
+  long long t0, t1;
+  // DFMA chain
+  t0 = clock64();
+  for (int i = 0; i < n; ++i) { a = fma(a, 0.999999, 1e-7); a = fma(a, 0.999999, 1e-7); a = fma(a, 0.999999, 1e-7); a = fma(a, 0.999999, 1e-7); }
+  t1 = clock64(); if (threadIdx.x == 0) cyc[0] = (t1 - t0);
+  // DADD chain
+  t0 = clock64();
+  for (int i = 0; i < n; ++i) { b = b + 1e-7; b = b + 1e-7; b = b + 1e-7; b = b + 1e-7; }
+  t1 = clock64(); if (threadIdx.x == 0) cyc[1] = (t1 - t0);
+  // MUFU.RSQ64H chain (+1 DADD to keep it positive and dependent)
+  double c = a;
+  t0 = clock64();
+  for (int i = 0; i < n; ++i) { double y; asm volatile("rsqrt.approx.ftz.f64 %0, %1;" : "=d"(y) : "d"(c)); c = y; }
+  t1 = clock64(); if (threadIdx.x == 0) cyc[2] = (t1 - t0);
+  // F2I + I2F chain-ish: F2I then IADD then use as LDS index
+  double d = a;
+  t0 = clock64();
+  for (int i = 0; i < n; ++i) { unsigned k = __double2uint_rz(d); double2 e = sm[k & 255]; d = e.x; }
+  t1 = clock64(); if (threadIdx.x == 0) cyc[3] = (t1 - t0);
+  // LDS.128 chain via integer index
+  t0 = clock64();
+  for (int i = 0; i < n; ++i) { double2 e = sm[u & 255]; u = __double_as_longlong(e.y) >> 40; u += (unsigned)__double_as_longlong(e.x); }
+  t1 = clock64(); if (threadIdx.x == 0) cyc[4] = (t1 - t0);
+  // IMAD.WIDE chain
+  unsigned long long w = u | 1;
+  t0 = clock64();
+  for (int i = 0; i < n; ++i) { w = w * 1220703125ull; w = w * 1220703125ull; w = w * 1220703125ull; w = w * 1220703125ull; }
+  t1 = clock64(); if (threadIdx.x == 0) cyc[5] = (t1 - t0);
+  out[threadIdx.x] = a + b + c + d + (double)u + (double)w;
+}
+
 int main() {
   cudaDeviceProp p;
   CK(cudaGetDeviceProperties(&p, 0));
@@ -79,6 +118,17 @@ int main() {
       printf("DFMA threads=%d blocks/SM=%d : %.2f lane-FMA/clk/SM (clock64), %.2f TFLOP/s, ms=%.3f, implied MHz=%.0f\n",
              threads, bps, lanes_per_clk_sm, tflops, ms, cmax / (ms * 1e3));
     }
+  }
+  {
+    long long* dc; double* dd;
+    CK(cudaMalloc(&dc, 64)); CK(cudaMalloc(&dd, 8 * 1024));
+    const int n = 4096;
+    lat_kernel<<<1, 32>>>(dd, dc, 1.5, n);
+    CK(cudaDeviceSynchronize());
+    long long hc[8];
+    CK(cudaMemcpy(hc, dc, 48, cudaMemcpyDeviceToHost));
+    printf("latency (cycles/dep op): DFMA %.2f  DADD %.2f  MUFU.RSQ64H %.2f  F2I+LDS %.2f  LDS.128+int %.2f  64b-mul %.2f\n",
+           hc[0] / (4.0 * n), hc[1] / (4.0 * n), hc[2] / double(n), hc[3] / double(n), hc[4] / double(n), hc[5] / (4.0 * n));
   }
   // approximation accuracy
   const int n = 1 << 22;
