@@ -45,7 +45,7 @@ ALG_OPS_ACCEPTED = 19
 P_ACCEPT = 0.7853981633974483
 ALG_OPS_PER_PAIR = ALG_OPS_ALWAYS + P_ACCEPT * ALG_OPS_ACCEPTED
 FP64_LANES_PER_SM_CLK = 64          # measured: tools/probe_fp64.cu (63.9-64.1 lane-DFMA/clk/SM)
-EP_PARAM_BYTES = 440                 # EPParams kernel-parameter block (jump table + scalars)
+EP_PARAM_BYTES = 560                 # EPParams kernel-parameter block (jump table, a^k table, coefs, scalars)
 
 
 def peaks():

@@ -36,13 +36,18 @@ def _stale() -> bool:
     return any(os.path.getmtime(p) > t for p in SOURCES + HEADERS + [__file__])
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not _stale():
+def build(force: bool = False, verbose: bool = False, out: str | None = None,
+          defines: tuple = ()) -> str:
+    """Compile libhpl.so.  `out`/`defines` build development A/B variants
+    (e.g. defines=("EP_ILP=4",)) to another path; the product is LIB."""
+    lib = out or LIB
+    if out is None and not defines and not force and not _stale():
         return LIB
-    tmp = LIB + ".tmp%d" % os.getpid()
-    cmd = [NVCC, *NVCC_FLAGS, "-I", os.path.join(ROOT, "include"), "-o", tmp, *SOURCES]
+    tmp = lib + ".tmp%d" % os.getpid()
+    cmd = [NVCC, *NVCC_FLAGS, *["-D" + d for d in defines], "-I", os.path.join(ROOT, "include"),
+           "-o", tmp, *SOURCES]
     res = subprocess.run(cmd, capture_output=True, text=True)
-    log = os.path.join(PKG, "build.log")
+    log = os.path.join(PKG, "build.log" if out is None else os.path.basename(lib) + ".log")
     with open(log, "w") as f:
         f.write(" ".join(cmd) + "\n" + res.stdout + res.stderr)
     if res.returncode != 0:
@@ -50,8 +55,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
         raise RuntimeError("nvcc failed (see %s)" % log)
     if verbose:
         sys.stderr.write(res.stderr)
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, lib)
+    return lib
 
 
 if __name__ == "__main__":

@@ -44,7 +44,7 @@ constexpr int LOG_K = 8;                       // mantissa bits per exponent
 constexpr int LOG_EMIN = -16;                  // table covers t >= ~2^LOG_EMIN
 constexpr int LOG_SHIFT = 20 - LOG_K;          // hi-word shift to the index
 constexpr uint32_t LOG_BIAS_TOP = 1023 - 2;    // biased exponent of t' = 1/4
-constexpr uint32_t LOG_IDX_MIN = uint32_t(LOG_BIAS_TOP + LOG_EMIN) << LOG_K;
+constexpr uint32_t LOG_IDX_MIN = uint32_t(int(LOG_BIAS_TOP) + LOG_EMIN) << LOG_K;
 constexpr uint32_t LOG_IDX_MAX = uint32_t(LOG_BIAS_TOP) << LOG_K;  // bucket of t' = 1/4
 constexpr uint32_t LOG_N = LOG_IDX_MAX - LOG_IDX_MIN + 1;  // 4097 real entries
 // u = (hi(t') + LOG_ADD) >> LOG_SHIFT  (mod 2^32), valid iff u < LOG_N
@@ -71,6 +71,7 @@ struct EPParams {
   double coef[6];        // lean constants (kept in the parameter bank, not registers)
   uint64_t a;            // multiplier
   unsigned a_lo, a_hi;   // its 32-bit halves
+  unsigned apow_lo[8], apow_hi[8];  // a^(k+1) mod 2^46, k = 0..7 (parallel LCG steps)
   uint64_t x_begin;      // state before the first uniform of this launch's range
   uint64_t npairs;       // pairs in this launch
   uint64_t base;         // pairs per thread (floor)

@@ -47,10 +47,35 @@ __device__ __forceinline__ double rsqrt_approx(double p) {
 
 // 1 << (8 l) for l in 0..3 in one PRMT (backward-4-extract of the byte string
 // {1,0,0,0,0,0,0,0} starting at byte l); lanes with l >= 4 never use it.
-__device__ __forceinline__ unsigned bin_increment(unsigned l) {
+__device__ __forceinline__ unsigned bin_increment(unsigned l, unsigned one = 1u) {
   unsigned r;
-  asm("prmt.b32.b4e %0, %1, %2, %3;" : "=r"(r) : "r"(1u), "r"(0u), "r"(l));
+  asm("prmt.b32.b4e %0, %1, %2, %3;" : "=r"(r) : "r"(one), "r"(0u), "r"(l));
   return r;
+}
+
+#ifndef EP_BIN_MODE
+#define EP_BIN_MODE 0  // 0: two F2I; 1: hi-word max + one F2I; 2: hi-word max + integer shift (no XU)
+#endif
+// l = trunc(max(|X|,|Y|)) for the common case, and ge4 = (max(|X|,|Y|) >= 4).
+// Modes 1/2 take the max on the high words: (hi << 1) drops the sign and
+// keeps the magnitude order, and for values < 2^20 the integer part depends
+// on the high word only, so no rounding question arises.  Mode 2 then
+// truncates with integer ops: (1.f) 2^21 >> (21 - e), e = exponent.
+__device__ __forceinline__ unsigned bin_index(double X, double Y, bool& ge4, unsigned implicit_bit) {
+  if (EP_BIN_MODE == 0) {
+    const unsigned l = max(__double2uint_rz(fabs(X)), __double2uint_rz(fabs(Y)));
+    ge4 = l >= 4;
+    return l;
+  }
+  const unsigned hx = static_cast<unsigned>(__double2hiint(X)) << 1;
+  const unsigned hy = static_cast<unsigned>(__double2hiint(Y)) << 1;
+  const unsigned m2 = max(hx, hy);
+  ge4 = m2 >= (0x40100000u << 1);
+  if (EP_BIN_MODE == 1) return __double2uint_rz(__hiloint2double(int(m2 >> 1), 0));
+  unsigned mn, l;
+  asm("lop3.b32 %0, %1, 0x1FFFFF, %2, 0xEA;" : "=r"(mn) : "r"(m2), "r"(implicit_bit));  // (m2 & 0x1FFFFF) | 2^21
+  asm("shr.b32 %0, %1, %2;" : "=r"(l) : "r"(mn), "r"(1044u - (m2 >> 21)));           // shift >= 32 -> 0
+  return l;
 }
 
 // One LCG step on the (lo, hi) words of v = bits(1 + x 2^-46):
@@ -63,6 +88,32 @@ __device__ __forceinline__ void lcg_step(unsigned& lo, unsigned& hi, unsigned a_
   hi = (ph & 0x000FFFFFu) | 0x3FF00000u;
 }
 
+
+// -2 ln(1+r) = r (-2 + r (1 + r (-2/3 + r (1/2 + r (c5 + r c6))))), |r| <= 2^-9.
+// c5 = -2/5 and c6 = 1/3 only weigh r^5, r^6 terms (< 2^-36 relative), so they
+// are rounded to 20-bit mantissas that encode as DFMA immediates (relative
+// effect < 2^-60); -2/3 stays exact (kernel parameter).  DESIGN.md §4.2.
+#define EP_C6 0x1.55555p-2    /* 1/3  rounded to 20 bits */
+#define EP_C5 -0x1.9999ap-2   /* -2/5 rounded to 20 bits */
+
+// Loop-invariant operands made opaque (asm volatile), so ptxas keeps them in
+// registers instead of rematerialising them with IMAD.MOV every iteration
+// (IMAD-pipe work contends with the FP64 pipe on sm_100).
+struct LeanConst {
+  double c6, c0375;
+  unsigned one, implicit_bit;
+};
+// `kc` is a shared-memory copy of {c6, 0.375, 1} written at kernel start; the
+// values are read back through asm volatile loads, which ptxas can neither
+// constant-fold nor duplicate.
+__device__ __forceinline__ LeanConst make_lean_const(unsigned kc) {
+  LeanConst K;
+  asm volatile("ld.shared.f64 %0, [%1];" : "=d"(K.c6) : "r"(kc));
+  asm volatile("ld.shared.f64 %0, [%1];" : "=d"(K.c0375) : "r"(kc + 8u));
+  asm volatile("ld.shared.u32 %0, [%1];" : "=r"(K.one) : "r"(kc + 16u));
+  asm volatile("ld.shared.u32 %0, [%1];" : "=r"(K.implicit_bit) : "r"(kc + 20u));
+  return K;
+}
 
 struct PairAcc {
   double csx, csy;
@@ -114,20 +165,20 @@ __device__ __forceinline__ void lean_pair(unsigned& vlo, unsigned& vhi, const EP
   const unsigned H = static_cast<unsigned>(__double2hiint(t));
   const unsigned u = min((H + LOG_ADD) >> LOG_SHIFT, LOG_N);
   double eT, eInv;
-  asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(eT), "=d"(eInv) : "r"(tab + u * 16u));
+  asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(eT), "=d"(eInv) : "r"((u << 4) + tab));
   const double r = fma(t, eInv, -1.0);
-  double c = fma(P.coef[0], r, P.coef[1]);
+  double c = fma(r, EP_C6, EP_C5);
   c = fma(c, r, 0.5);
   c = fma(c, r, P.coef[2]);
   c = fma(c, r, 1.0);
   c = fma(c, r, -2.0);
   const double L = fma(c, r, eT);
   // t2' = sqrt(L/t) = L rsqrt(L t): MUFU seed + one cubic Newton step
-  const double p = fma(L, t, P.coef[5]);  // + 2^-200: t' == 1/4 -> L = 0 -> t2' = 0
+  const double p = fma(L, t, 0x1p-200);  // + 2^-200: t' == 1/4 -> L = 0 -> t2' = 0
   const double y0 = rsqrt_approx(p);
   const double h = __dmul_rn(p, y0);
   const double e = fma(-h, y0, 1.0);
-  const double cc = fma(e, P.coef[3], 0.5);
+  const double cc = fma(e, 0.375, 0.5);
   const double g = __dmul_rn(L, y0);
   const double ge = __dmul_rn(g, e);
   const double t2 = fma(ge, cc, g);
@@ -146,6 +197,209 @@ __device__ __forceinline__ void lean_pair(unsigned& vlo, unsigned& vhi, const EP
     A.csx += o.dx;
     A.csy += o.dy;
     A.cnt += o.dcnt;
+  }
+}
+
+// W consecutive pairs in lockstep (stage by stage), so that the W independent
+// dependency chains interleave in the instruction stream (ILP W) while the
+// LCG chain between them stays short.  One rare-path branch per group.
+#ifndef EP_ACC_INT
+#define EP_ACC_INT 1   // 1: acceptance t' <= 1/4 by a 64-bit integer compare of the bits
+#endif
+#ifndef EP_LCG_PAR
+#define EP_LCG_PAR 0   // 1: the 2W uniforms of a group from v by independent a^k multiplies
+#endif
+#ifndef EP_ILP
+#define EP_ILP 2       // pairs in lockstep for the 85..128-register tiers
+#endif
+
+template <bool A32, int W>
+__device__ __forceinline__ void lean_pairs(unsigned& vlo, unsigned& vhi, const EPParams& P,
+                                           unsigned tab, PairAcc& A, unsigned long long* s_rare) {
+  double x1[W], x2[W], t[W], X[W], Y[W];
+  unsigned u[W], l[W];
+  bool acc[W], ok[W];
+  if (EP_LCG_PAR) {
+    // v_k = a^k v_0 mod 2^52 (| bits(1.0)), k = 1..2W: one multiply deep
+    const unsigned lo0 = vlo, hi0 = vhi;
+#pragma unroll
+    for (int k = 0; k < 2 * W; ++k) {
+      const unsigned alo = P.apow_lo[k], ahi = P.apow_hi[k];
+      const unsigned ph = __umulhi(lo0, alo) + hi0 * alo + lo0 * ahi;
+      const unsigned hi = (ph & 0x000FFFFFu) | 0x3FF00000u;
+      const double v = __hiloint2double(int(hi), int(lo0 * alo));
+      if (k & 1) x2[k >> 1] = __dadd_rn(v, -1.5);
+      else x1[k >> 1] = __dadd_rn(v, -1.5);
+      if (k == 2 * W - 1) { vlo = lo0 * alo; vhi = hi; }
+    }
+  } else {
+#pragma unroll
+    for (int k = 0; k < W; ++k) {
+      lcg_step<A32>(vlo, vhi, P.a_lo, P.a_hi);
+      x1[k] = __dadd_rn(__hiloint2double(int(vhi), int(vlo)), -1.5);
+      lcg_step<A32>(vlo, vhi, P.a_lo, P.a_hi);
+      x2[k] = __dadd_rn(__hiloint2double(int(vhi), int(vlo)), -1.5);
+    }
+  }
+#pragma unroll
+  for (int k = 0; k < W; ++k) {
+    t[k] = __dadd_rn(__dmul_rn(x1[k], x1[k]), __dmul_rn(x2[k], x2[k]));
+    if (EP_ACC_INT)
+      acc[k] = static_cast<unsigned long long>(__double_as_longlong(t[k])) <= 0x3FD0000000000000ull;
+    else
+      acc[k] = t[k] <= 0.25;
+    u[k] = min((static_cast<unsigned>(__double2hiint(t[k])) + LOG_ADD) >> LOG_SHIFT, LOG_N);
+  }
+  double eT[W], eInv[W];
+#pragma unroll
+  for (int k = 0; k < W; ++k)
+    asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(eT[k]), "=d"(eInv[k]) : "r"((u[k] << 4) + tab));
+  double r[W], c[W], L[W];
+#pragma unroll
+  for (int k = 0; k < W; ++k) {
+    r[k] = fma(t[k], eInv[k], -1.0);
+    c[k] = fma(r[k], EP_C6, EP_C5);
+  }
+#pragma unroll
+  for (int k = 0; k < W; ++k) c[k] = fma(c[k], r[k], 0.5);
+#pragma unroll
+  for (int k = 0; k < W; ++k) c[k] = fma(c[k], r[k], P.coef[2]);
+#pragma unroll
+  for (int k = 0; k < W; ++k) c[k] = fma(c[k], r[k], 1.0);
+#pragma unroll
+  for (int k = 0; k < W; ++k) c[k] = fma(c[k], r[k], -2.0);
+#pragma unroll
+  for (int k = 0; k < W; ++k) L[k] = fma(c[k], r[k], eT[k]);
+  double p[W], y0[W], e[W], g[W], t2[W];
+#pragma unroll
+  for (int k = 0; k < W; ++k) {
+    p[k] = fma(L[k], t[k], 0x1p-200);
+    y0[k] = rsqrt_approx(p[k]);
+  }
+#pragma unroll
+  for (int k = 0; k < W; ++k) e[k] = fma(-__dmul_rn(p[k], y0[k]), y0[k], 1.0);
+#pragma unroll
+  for (int k = 0; k < W; ++k) {
+    g[k] = __dmul_rn(L[k], y0[k]);
+    t2[k] = fma(__dmul_rn(g[k], e[k]), fma(e[k], 0.375, 0.5), g[k]);
+  }
+  bool any_rare = false;
+#pragma unroll
+  for (int k = 0; k < W; ++k) {
+    X[k] = __dmul_rn(x1[k], t2[k]);
+    Y[k] = __dmul_rn(x2[k], t2[k]);
+    l[k] = max(__double2uint_rz(fabs(X[k])), __double2uint_rz(fabs(Y[k])));
+    ok[k] = acc[k] && l[k] < 4;
+    if (ok[k]) {
+      A.csx = __dadd_rn(A.csx, X[k]);
+      A.csy = __dadd_rn(A.csy, Y[k]);
+      A.cnt += bin_increment(l[k]);
+    }
+    any_rare |= acc[k] && !ok[k];
+  }
+  if (any_rare) {
+#pragma unroll
+    for (int k = 0; k < W; ++k)
+      if (acc[k] && !ok[k]) {
+        const RareOut o = rare_pair(t[k], x1[k], x2[k], X[k], Y[k], u[k], s_rare);
+        A.csx += o.dx;
+        A.csy += o.dy;
+        A.cnt += o.dcnt;
+      }
+  }
+}
+
+#ifndef EP_PIPE
+#define EP_PIPE 1      // 1: software-pipeline generation of group g+1 under the transform of group g
+#endif
+
+// Software-pipelined form of lean_pairs: gen_stage produces the LCG pairs, t',
+// the table index and the table entries of a group (integer + LDS heavy);
+// transform_stage consumes them (FP64 heavy).  The main loop ping-pongs two
+// stages so each transform is interleaved with the next group's generation.
+template <int W>
+struct Stage {
+  double x1[W], x2[W], t[W], eT[W], eInv[W];
+  unsigned u[W];
+};
+
+template <bool A32, int W>
+__device__ __forceinline__ void gen_stage(unsigned& vlo, unsigned& vhi, const EPParams& P, unsigned tab,
+                                          Stage<W>& S) {
+#pragma unroll
+  for (int k = 0; k < W; ++k) {
+    lcg_step<A32>(vlo, vhi, P.a_lo, P.a_hi);
+    S.x1[k] = __dadd_rn(__hiloint2double(int(vhi), int(vlo)), -1.5);
+    lcg_step<A32>(vlo, vhi, P.a_lo, P.a_hi);
+    S.x2[k] = __dadd_rn(__hiloint2double(int(vhi), int(vlo)), -1.5);
+  }
+#pragma unroll
+  for (int k = 0; k < W; ++k) {
+    S.t[k] = __dadd_rn(__dmul_rn(S.x1[k], S.x1[k]), __dmul_rn(S.x2[k], S.x2[k]));
+    S.u[k] = min((static_cast<unsigned>(__double2hiint(S.t[k])) + LOG_ADD) >> LOG_SHIFT, LOG_N);
+  }
+#pragma unroll
+  for (int k = 0; k < W; ++k)
+    asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(S.eT[k]), "=d"(S.eInv[k]) : "r"((S.u[k] << 4) + tab));
+}
+
+template <int W>
+__device__ __forceinline__ void transform_stage(const Stage<W>& S, const EPParams& P, const LeanConst& K,
+                                                PairAcc& A, unsigned long long* s_rare) {
+  double r[W], c[W], L[W], p[W], y0[W], e[W], g[W], t2[W], X[W], Y[W];
+  unsigned l[W];
+  bool acc[W], ok[W];
+#pragma unroll
+  for (int k = 0; k < W; ++k) {
+    if (EP_ACC_INT)
+      acc[k] = static_cast<unsigned long long>(__double_as_longlong(S.t[k])) <= 0x3FD0000000000000ull;
+    else
+      acc[k] = S.t[k] <= 0.25;
+    r[k] = fma(S.t[k], S.eInv[k], -1.0);
+    c[k] = fma(r[k], K.c6, EP_C5);
+  }
+#pragma unroll
+  for (int k = 0; k < W; ++k) c[k] = fma(c[k], r[k], 0.5);
+#pragma unroll
+  for (int k = 0; k < W; ++k) c[k] = fma(c[k], r[k], P.coef[2]);
+#pragma unroll
+  for (int k = 0; k < W; ++k) c[k] = fma(c[k], r[k], 1.0);
+#pragma unroll
+  for (int k = 0; k < W; ++k) c[k] = fma(c[k], r[k], -2.0);
+#pragma unroll
+  for (int k = 0; k < W; ++k) {
+    L[k] = fma(c[k], r[k], S.eT[k]);
+    p[k] = fma(L[k], S.t[k], 0x1p-200);
+    y0[k] = rsqrt_approx(p[k]);
+  }
+#pragma unroll
+  for (int k = 0; k < W; ++k) e[k] = fma(-__dmul_rn(p[k], y0[k]), y0[k], 1.0);
+  bool any_rare = false;
+#pragma unroll
+  for (int k = 0; k < W; ++k) {
+    g[k] = __dmul_rn(L[k], y0[k]);
+    t2[k] = fma(__dmul_rn(g[k], e[k]), fma(e[k], K.c0375, 0.5), g[k]);
+    X[k] = __dmul_rn(S.x1[k], t2[k]);
+    Y[k] = __dmul_rn(S.x2[k], t2[k]);
+    bool ge4;
+    l[k] = bin_index(X[k], Y[k], ge4, K.implicit_bit);
+    ok[k] = acc[k] && !ge4;
+    if (ok[k]) {
+      A.csx = __dadd_rn(A.csx, X[k]);
+      A.csy = __dadd_rn(A.csy, Y[k]);
+      A.cnt += bin_increment(l[k], K.one);
+    }
+    any_rare |= acc[k] && !ok[k];
+  }
+  if (any_rare) {
+#pragma unroll
+    for (int k = 0; k < W; ++k)
+      if (acc[k] && !ok[k]) {
+        const RareOut o = rare_pair(S.t[k], S.x1[k], S.x2[k], X[k], Y[k], S.u[k], s_rare);
+        A.csx += o.dx;
+        A.csy += o.dy;
+        A.cnt += o.dcnt;
+      }
   }
 }
 
@@ -171,24 +425,32 @@ __device__ __forceinline__ void libdevice_pair(unsigned& vlo, unsigned& vhi, con
   }
 }
 
-template <int VARIANT, bool A32, int NT, int MINB>
+template <int VARIANT, bool A32, int NT, int MINB, int W>
 __global__ void __launch_bounds__(NT, MINB)
 ep_kernel(const __grid_constant__ EPParams P) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   __shared__ unsigned long long s_rare[7];  // bins 4..9, then l >= 10
+  __shared__ double s_kc[3];                // LeanConst source (see make_lean_const)
   __shared__ double s_wsx[EP_MAX_THREADS / 32], s_wsy[EP_MAX_THREADS / 32];
   __shared__ unsigned long long s_wq[EP_MAX_THREADS / 32][4];
   __shared__ int s_last;
   __shared__ double s_fin[13];
 
   const unsigned tid = threadIdx.x;
-  const unsigned tab = static_cast<unsigned>(__cvta_generic_to_shared(smem_raw));
+  unsigned tab;  // opaque copy: keeps the shared base in a register (no per-use rematerialisation)
+  asm volatile("mov.u32 %0, %1;" : "=r"(tab) : "r"(static_cast<unsigned>(__cvta_generic_to_shared(smem_raw))));
   if (VARIANT == HPL_VARIANT_LEAN) {
     const double2* src = reinterpret_cast<const double2*>(P.table);
     double2* dst = reinterpret_cast<double2*>(smem_raw);
     for (unsigned i = tid; i < LOG_TAB; i += blockDim.x) dst[i] = __ldg(src + i);
   }
   if (tid < 7) s_rare[tid] = 0;
+  if (tid == 0) {
+    s_kc[0] = EP_C6;
+    s_kc[1] = 0.375;
+    reinterpret_cast<unsigned*>(s_kc)[4] = 1u;
+    reinterpret_cast<unsigned*>(s_kc)[5] = 0x200000u;
+  }
   __syncthreads();
 
   // ---- A2: this thread's pair range and start state
@@ -208,29 +470,63 @@ ep_kernel(const __grid_constant__ EPParams P) {
     sx += A.csx;
     sy += A.csy;
   };
-  // 8-bit packed counters overflow after 255 pairs: chunks of 252 = 63 x 4
-  constexpr unsigned UNROLL = 4, CHUNK = 63 * UNROLL;
-  uint64_t rem = n_t;
-  for (; rem >= CHUNK; rem -= CHUNK) {
-    PairAcc A{0.0, 0.0, 0u};
+  if (VARIANT == HPL_VARIANT_LEAN && EP_PIPE) {
+    // 8-bit packed counters overflow after 255 pairs: <= 252 pairs per flush.
+    // Tail pairs first, so the pipelined loop's one-group overshoot past the
+    // thread's range is never transformed.
+    constexpr unsigned PER_IT = 2 * W, IT_PER_CHUNK = 252 / PER_IT;
+    const unsigned tail = unsigned(n_t % PER_IT);
+    if (tail) {
+      PairAcc A{0.0, 0.0, 0u};
 #pragma unroll 1
-    for (unsigned i = 0; i < CHUNK / UNROLL; ++i) {
-#pragma unroll
-      for (unsigned j = 0; j < UNROLL; ++j) {
+      for (unsigned i = 0; i < tail; ++i) lean_pair<A32>(vlo, vhi, P, tab, A, s_rare);
+      flush(A);
+    }
+    uint64_t iters = n_t / PER_IT;
+    const LeanConst K = make_lean_const(static_cast<unsigned>(__cvta_generic_to_shared(s_kc)));
+    Stage<W> s0, s1;
+    if (iters) gen_stage<A32, W>(vlo, vhi, P, tab, s0);
+    while (iters) {
+      const unsigned ci = iters < IT_PER_CHUNK ? unsigned(iters) : IT_PER_CHUNK;
+      PairAcc A{0.0, 0.0, 0u};
+#pragma unroll 1
+      for (unsigned i = 0; i < ci; ++i) {
+        gen_stage<A32, W>(vlo, vhi, P, tab, s1);
+        transform_stage<W>(s0, P, K, A, s_rare);
+        gen_stage<A32, W>(vlo, vhi, P, tab, s0);
+        transform_stage<W>(s1, P, K, A, s_rare);
+      }
+      flush(A);
+      iters -= ci;
+    }
+  } else {
+    // 8-bit packed counters overflow after 255 pairs: chunks of 252 = 63 x 4
+    constexpr unsigned UNROLL = 4, CHUNK = 63 * UNROLL;
+    static_assert(UNROLL % W == 0, "W must divide UNROLL");
+    uint64_t rem = n_t;
+    for (; rem >= CHUNK; rem -= CHUNK) {
+      PairAcc A{0.0, 0.0, 0u};
+  #pragma unroll 1
+      for (unsigned i = 0; i < CHUNK / UNROLL; ++i) {
+        if (VARIANT == HPL_VARIANT_LEAN) {
+  #pragma unroll
+          for (unsigned j = 0; j < UNROLL / W; ++j) lean_pairs<A32, W>(vlo, vhi, P, tab, A, s_rare);
+        } else {
+  #pragma unroll
+          for (unsigned j = 0; j < UNROLL; ++j) libdevice_pair<A32>(vlo, vhi, P, tab, A, s_rare);
+        }
+      }
+      flush(A);
+    }
+    if (rem) {
+      PairAcc A{0.0, 0.0, 0u};
+  #pragma unroll 1
+      for (unsigned i = 0; i < unsigned(rem); ++i) {
         if (VARIANT == HPL_VARIANT_LEAN) lean_pair<A32>(vlo, vhi, P, tab, A, s_rare);
         else libdevice_pair<A32>(vlo, vhi, P, tab, A, s_rare);
       }
+      flush(A);
     }
-    flush(A);
-  }
-  if (rem) {
-    PairAcc A{0.0, 0.0, 0u};
-#pragma unroll 1
-    for (unsigned i = 0; i < unsigned(rem); ++i) {
-      if (VARIANT == HPL_VARIANT_LEAN) lean_pair<A32>(vlo, vhi, P, tab, A, s_rare);
-      else libdevice_pair<A32>(vlo, vhi, P, tab, A, s_rare);
-    }
-    flush(A);
   }
 
   // ---- A8: warp -> block reduction (fixed order => deterministic)
@@ -318,11 +614,13 @@ __global__ void lcg_states_kernel(uint64_t seed, uint64_t a, uint64_t offset, ui
 using EPKernel = void (*)(const EPParams);
 template <int V, bool A32>
 static EPKernel tier_kernel(int thr) {
-  if (thr <= 128) return ep_kernel<V, A32, 128, 4>;
-  if (thr <= 256) return ep_kernel<V, A32, 256, 3>;
-  if (thr <= 384) return ep_kernel<V, A32, 384, 2>;
-  if (thr <= 512) return ep_kernel<V, A32, 512, 2>;
-  return ep_kernel<V, A32, 1024, 1>;
+  if (thr <= 128) return ep_kernel<V, A32, 128, 4, 1>;   // 128 regs
+  if (thr <= 256) return ep_kernel<V, A32, 256, 3, EP_ILP>;   //  85 regs
+  if (thr <= 384) return ep_kernel<V, A32, 384, 2, EP_ILP>;   //  85 regs
+  if (thr <= 512) return ep_kernel<V, A32, 512, 1, EP_ILP>;   // 128 regs
+  if (thr <= 640) return ep_kernel<V, A32, 640, 1, EP_ILP>;   // 102 regs
+  if (thr <= 768) return ep_kernel<V, A32, 768, 1, EP_ILP>;   //  85 regs
+  return ep_kernel<V, A32, 1024, 1, 1>;                  //  64 regs
 }
 static EPKernel pick_kernel(int variant, bool a32, int thr) {
   if (variant == HPL_VARIANT_LEAN) return a32 ? tier_kernel<HPL_VARIANT_LEAN, true>(thr) : tier_kernel<HPL_VARIANT_LEAN, false>(thr);
@@ -382,7 +680,7 @@ int set_attrs_once(int device) {
   if ((int)done.size() <= device) done.resize(device + 1, 0);
   if (done[device]) return 0;
   const int smem = int(LOG_TAB * sizeof(LogEntry));
-  for (int thr : {128, 256, 384, 512, 1024})
+  for (int thr : {128, 256, 384, 512, 640, 768, 1024})
     for (bool a32 : {true, false}) {
       cudaError_t e = cudaFuncSetAttribute(pick_kernel(HPL_VARIANT_LEAN, a32, thr),
                                            cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
@@ -497,6 +795,14 @@ int launch_ep(int device, uint64_t seed, uint64_t a, uint64_t pair_begin, uint64
   P.a = a;
   P.a_lo = unsigned(a);
   P.a_hi = unsigned(a >> 32);
+  {
+    uint64_t ak = a & MASK46;
+    for (int k = 0; k < 8; ++k) {  // a^(k+1) mod 2^46
+      P.apow_lo[k] = unsigned(ak);
+      P.apow_hi[k] = unsigned(ak >> 32);
+      ak = mulmod46(ak, a);
+    }
+  }
   const double coef[6] = {1.0 / 3.0, -0.4, -2.0 / 3.0, 0.375, 0.5, 0x1p-200};
   for (int i = 0; i < 6; ++i) P.coef[i] = coef[i];
   P.x_begin = host_jump(seed & MASK46, 2 * pair_begin, P.jump);

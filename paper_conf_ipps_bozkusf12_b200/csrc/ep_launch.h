@@ -12,7 +12,7 @@ namespace hplep {
 
 constexpr int HPL_VARIANT_LEAN = HPL_EP_LEAN;
 constexpr int HPL_VARIANT_LIBDEVICE = HPL_EP_LIBDEVICE;
-constexpr int EP_DEFAULT_THREADS = 1024;
+constexpr int EP_DEFAULT_THREADS = 512;
 constexpr uint64_t EP_MIN_PAIRS_PER_THREAD = 64;
 
 struct EPConfig {

@@ -15,7 +15,8 @@ import ctypes
 import os
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libhpl.so")
+# HPL_LIB: development override to load an A/B build variant of the library
+LIB_PATH = os.environ.get("HPL_LIB") or os.path.join(_PKG, "libhpl.so")
 
 HPL_OK, HPL_EINVAL, HPL_ENOMEM, HPL_ECUDA, HPL_ENODEV, HPL_ERANGE, HPL_ESTATE = 0, -1, -2, -3, -4, -5, -6
 HPL_F64, HPL_F32, HPL_U64, HPL_I64, HPL_I32, HPL_U32 = 0, 1, 2, 3, 4, 5

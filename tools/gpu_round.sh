@@ -15,6 +15,10 @@ bench)
   timeout 600 python bench.py > gpurun_out/${TAG}_bench.json 2> gpurun_out/${TAG}_bench.err; cat gpurun_out/${TAG}_bench.json ;;
 ref)
   timeout 600 python bench.py --impl reference > gpurun_out/${TAG}_ref.json 2> gpurun_out/${TAG}_ref.err; cat gpurun_out/${TAG}_ref.json ;;
+probe)
+  nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o tools/probe_fp64 tools/probe_fp64.cu && ./tools/probe_fp64 > gpurun_out/${TAG}_probe.log 2>&1; cat gpurun_out/${TAG}_probe.log ;;
+qt)
+  python tools/quick_time.py 32 36 --threads ${QT_THREADS:-1024} > gpurun_out/${TAG}_qt.log 2>&1; cat gpurun_out/${TAG}_qt.log ;;
 ncu)
   timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${TAG}_launches.csv \
       python bench.py --steps 2 --warmup 3 --no-cpu-baseline > gpurun_out/${TAG}_ncu_bench.log 2>&1

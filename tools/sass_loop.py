@@ -3,8 +3,8 @@
 python tools/sass_loop.py [kernel-substring] — finds the largest backward
 branch loop in the kernel and counts instructions per pipe class per pair.
 """
-import re, subprocess, sys, collections
-lib = "paper_conf_ipps_bozkusf12_b200/libhpl.so"
+import os, re, subprocess, sys, collections
+lib = os.environ.get("HPL_LIB", "paper_conf_ipps_bozkusf12_b200/libhpl.so")
 pat = sys.argv[1] if len(sys.argv) > 1 else "ep_kernelILi0ELb1"
 unroll = int(sys.argv[2]) if len(sys.argv) > 2 else 4
 out = subprocess.run(["cuobjdump", "-sass", lib], capture_output=True, text=True).stdout
@@ -27,7 +27,15 @@ for addr, ins in lines:
             if n >= unroll and (best is None or addr - tgt < best[1] - best[0]):
                 best = (tgt, addr)
 lo, hi = best
-body = [ins for a, ins in lines if lo <= a <= hi]
+# cold regions: bodies of forward conditional branches that contain a CALL (rare path)
+cold = []
+for a, ins in lines:
+    m = re.search(r"^@!?U?P\w+\s+BRA (?:!?U?P\d, )?0x([0-9a-f]+)", ins)
+    if m and lo <= a <= hi:
+        t = int(m.group(1), 16)
+        if t > a and any("CALL" in i for b, i in lines if a < b < t):
+            cold.append((a, t))
+body = [ins for a, ins in lines if lo <= a <= hi and not any(c0 < a < c1 for c0, c1 in cold)]
 def cls(i):
     op = re.sub(r"^@!?U?P\w+\s+", "", i).split()[0]
     base = op.split(".")[0]
