@@ -185,11 +185,17 @@ def run_ours(args, M):
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if world != args.gpus:
         raise SystemExit("--gpus %d but WORLD_SIZE=%d (launch with torchrun for N>1)" % (args.gpus, world))
-    torch.cuda.set_device(local)
-    hpl.hpl_set_device(local)
-    dev = torch.device("cuda", local)
+    # one rank per GPU; --dist-backend gloo lets several ranks share one GPU
+    # (code-path test on a 1-GPU box, never a performance number)
+    gpu = local % max(torch.cuda.device_count(), 1) if args.dist_backend == "gloo" else local
+    torch.cuda.set_device(gpu)
+    hpl.hpl_set_device(gpu)
+    dev = torch.device("cuda", gpu)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if args.dist_backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group("gloo")
     stream = torch.cuda.current_stream(dev)
     out = torch.empty(13, dtype=torch.float64, device=dev)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # > 126 MB L2
@@ -204,7 +210,7 @@ def run_ours(args, M):
     torch.cuda.synchronize(dev)
 
     # ---- device-timed region
-    sampler = ClockSampler(local)
+    sampler = ClockSampler(gpu)
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize(dev)
@@ -294,6 +300,7 @@ def run_ours(args, M):
                     "note": "h2d = kernel-parameter block (jump table + scalars); d2h = 13-word result"},
             "gpu_launches": launches_all,
             "clocks": clocks,
+            "dist_backend": args.dist_backend if world > 1 else None,
             "result": {"sx": result["sx"], "sy": result["sy"], "gc": result["gc"]},
         }
         if not args.no_cpu_baseline and world == 1:
@@ -315,6 +322,8 @@ def main():
     ap.add_argument("--cpu-budget", type=float, default=15.0, help="seconds of oracle work for cpu_baseline")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--ref-batches", type=int, default=0, help="NPB batches per --impl reference step")
+    ap.add_argument("--dist-backend", choices=["nccl", "gloo"], default="nccl",
+                    help="gloo only to exercise the N>1 code path with several ranks on one GPU")
     args = ap.parse_args()
     if args.warmup < 3:
         ap.error("--warmup must be >= 3")

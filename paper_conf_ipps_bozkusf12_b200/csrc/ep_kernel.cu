@@ -309,6 +309,9 @@ __device__ __forceinline__ void lean_pairs(unsigned& vlo, unsigned& vhi, const E
   }
 }
 
+#ifndef EP_KMODE
+#define EP_KMODE 0     // 1: loop constants as immediates + kernel-parameter (uniform) operands
+#endif
 #ifndef EP_PIPE
 #define EP_PIPE 1      // 1: software-pipeline generation of group g+1 under the transform of group g
 #endif
@@ -356,7 +359,13 @@ __device__ __forceinline__ void transform_stage(const Stage<W>& S, const EPParam
     else
       acc[k] = S.t[k] <= 0.25;
     r[k] = fma(S.t[k], S.eInv[k], -1.0);
+#if EP_KMODE == 1
+    c[k] = fma(r[k], EP_C6, P.coef[1]);  // c6 immediate (b slot), c5 uniform (param -> UR)
+#elif EP_KMODE == 2
+    c[k] = fma(r[k], P.coef[0], EP_C5);  // c6 uniform (param -> UR, b slot), c5 immediate
+#else
     c[k] = fma(r[k], K.c6, EP_C5);
+#endif
   }
 #pragma unroll
   for (int k = 0; k < W; ++k) c[k] = fma(c[k], r[k], 0.5);
@@ -378,7 +387,13 @@ __device__ __forceinline__ void transform_stage(const Stage<W>& S, const EPParam
 #pragma unroll
   for (int k = 0; k < W; ++k) {
     g[k] = __dmul_rn(L[k], y0[k]);
+#if EP_KMODE == 1
+    t2[k] = fma(__dmul_rn(g[k], e[k]), fma(e[k], 0.375, P.coef[4]), g[k]);
+#elif EP_KMODE == 2
+    t2[k] = fma(__dmul_rn(g[k], e[k]), fma(e[k], P.coef[3], 0.5), g[k]);
+#else
     t2[k] = fma(__dmul_rn(g[k], e[k]), fma(e[k], K.c0375, 0.5), g[k]);
+#endif
     X[k] = __dmul_rn(S.x1[k], t2[k]);
     Y[k] = __dmul_rn(S.x2[k], t2[k]);
     bool ge4;
@@ -614,10 +629,25 @@ __global__ void lcg_states_kernel(uint64_t seed, uint64_t a, uint64_t offset, ui
 using EPKernel = void (*)(const EPParams);
 template <int V, bool A32>
 static EPKernel tier_kernel(int thr) {
+#ifndef EP_T256_MINB
+#define EP_T256_MINB 3
+#endif
+#ifndef EP_T256_W
+#define EP_T256_W EP_ILP
+#endif
+#ifndef EP_T384_MINB
+#define EP_T384_MINB 2
+#endif
+#ifndef EP_T384_W
+#define EP_T384_W EP_ILP
+#endif
+#ifndef EP_T512_W
+#define EP_T512_W EP_ILP
+#endif
   if (thr <= 128) return ep_kernel<V, A32, 128, 4, 1>;   // 128 regs
-  if (thr <= 256) return ep_kernel<V, A32, 256, 3, EP_ILP>;   //  85 regs
-  if (thr <= 384) return ep_kernel<V, A32, 384, 2, EP_ILP>;   //  85 regs
-  if (thr <= 512) return ep_kernel<V, A32, 512, 1, EP_ILP>;   // 128 regs
+  if (thr <= 256) return ep_kernel<V, A32, 256, EP_T256_MINB, EP_T256_W>;   //  85 regs (3 blocks/SM)
+  if (thr <= 384) return ep_kernel<V, A32, 384, EP_T384_MINB, EP_T384_W>;   //  85 regs (2 blocks/SM)
+  if (thr <= 512) return ep_kernel<V, A32, 512, 1, EP_T512_W>;   // 128 regs
   if (thr <= 640) return ep_kernel<V, A32, 640, 1, EP_ILP>;   // 102 regs
   if (thr <= 768) return ep_kernel<V, A32, 768, 1, EP_ILP>;   //  85 regs
   return ep_kernel<V, A32, 1024, 1, 1>;                  //  64 regs
@@ -803,7 +833,7 @@ int launch_ep(int device, uint64_t seed, uint64_t a, uint64_t pair_begin, uint64
       ak = mulmod46(ak, a);
     }
   }
-  const double coef[6] = {1.0 / 3.0, -0.4, -2.0 / 3.0, 0.375, 0.5, 0x1p-200};
+  const double coef[6] = {EP_C6, EP_C5, -2.0 / 3.0, 0.375, 0.5, 0x1p-200};
   for (int i = 0; i < 6; ++i) P.coef[i] = coef[i];
   P.x_begin = host_jump(seed & MASK46, 2 * pair_begin, P.jump);
   P.npairs = npairs;

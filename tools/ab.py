@@ -1,6 +1,6 @@
 """A/B build variants of libhpl.so with -D switches (development aid).
 
-  python tools/ab.py build name=DEF1,DEF2 name2=...     (CPU: compile into build_ab/)
+  python tools/ab.py build "name=DEF1;DEF2" name2=...     (CPU: compile into build_ab/)
   python tools/ab.py time M threads [names...]          (GPU: time each variant)
 """
 import json, os, subprocess, sys
@@ -13,7 +13,7 @@ if sys.argv[1] == "build":
     os.makedirs(OUT, exist_ok=True)
     for spec in sys.argv[2:]:
         name, _, defs = spec.partition("=")
-        d = tuple(x for x in defs.split(",") if x)
+        d = tuple(x for x in defs.split(";") if x)
         build.build(out=os.path.join(OUT, "libhpl_%s.so" % name), defines=d)
         print("built", name, d)
 else:
