@@ -81,6 +81,16 @@ __device__ __forceinline__ unsigned bin_index(double X, double Y, bool& ge4, uns
 // One LCG step on the (lo, hi) words of v = bits(1 + x 2^-46):
 //   v' = ((a v) mod 2^52) | bits(1.0)
 // = IMAD.WIDE.U32 + IMAD (+ IMAD if a >= 2^32) + one LOP3 doing mask and OR.
+// Same step with bits(1.0)'s high word supplied in a register, so mask and
+// OR fuse into one LOP3 (ptxas otherwise splits them: two 32-bit constants).
+template <bool A32>
+__device__ __forceinline__ void lcg_step_k(unsigned& lo, unsigned& hi, unsigned a_lo, unsigned a_hi,
+                                           unsigned exp_hi) {
+  const unsigned ph = __umulhi(lo, a_lo) + hi * a_lo + (A32 ? 0u : lo * a_hi);
+  lo = lo * a_lo;
+  asm("lop3.b32 %0, %1, 0x000FFFFF, %2, 0xEA;" : "=r"(hi) : "r"(ph), "r"(exp_hi));
+}
+
 template <bool A32>
 __device__ __forceinline__ void lcg_step(unsigned& lo, unsigned& hi, unsigned a_lo, unsigned a_hi) {
   const unsigned ph = __umulhi(lo, a_lo) + hi * a_lo + (A32 ? 0u : lo * a_hi);
@@ -101,7 +111,7 @@ __device__ __forceinline__ void lcg_step(unsigned& lo, unsigned& hi, unsigned a_
 // (IMAD-pipe work contends with the FP64 pipe on sm_100).
 struct LeanConst {
   double c6, c0375;
-  unsigned one, implicit_bit;
+  unsigned one, implicit_bit, exp_hi;
 };
 // `kc` is a shared-memory copy of {c6, 0.375, 1} written at kernel start; the
 // values are read back through asm volatile loads, which ptxas can neither
@@ -112,6 +122,7 @@ __device__ __forceinline__ LeanConst make_lean_const(unsigned kc) {
   asm volatile("ld.shared.f64 %0, [%1];" : "=d"(K.c0375) : "r"(kc + 8u));
   asm volatile("ld.shared.u32 %0, [%1];" : "=r"(K.one) : "r"(kc + 16u));
   asm volatile("ld.shared.u32 %0, [%1];" : "=r"(K.implicit_bit) : "r"(kc + 20u));
+  asm volatile("ld.shared.u32 %0, [%1];" : "=r"(K.exp_hi) : "r"(kc + 24u));
   return K;
 }
 
@@ -328,12 +339,12 @@ struct Stage {
 
 template <bool A32, int W>
 __device__ __forceinline__ void gen_stage(unsigned& vlo, unsigned& vhi, const EPParams& P, unsigned tab,
-                                          Stage<W>& S) {
+                                          Stage<W>& S, unsigned exp_hi) {
 #pragma unroll
   for (int k = 0; k < W; ++k) {
-    lcg_step<A32>(vlo, vhi, P.a_lo, P.a_hi);
+    lcg_step_k<A32>(vlo, vhi, P.a_lo, P.a_hi, exp_hi);
     S.x1[k] = __dadd_rn(__hiloint2double(int(vhi), int(vlo)), -1.5);
-    lcg_step<A32>(vlo, vhi, P.a_lo, P.a_hi);
+    lcg_step_k<A32>(vlo, vhi, P.a_lo, P.a_hi, exp_hi);
     S.x2[k] = __dadd_rn(__hiloint2double(int(vhi), int(vlo)), -1.5);
   }
 #pragma unroll
@@ -445,7 +456,7 @@ __global__ void __launch_bounds__(NT, MINB)
 ep_kernel(const __grid_constant__ EPParams P) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   __shared__ unsigned long long s_rare[7];  // bins 4..9, then l >= 10
-  __shared__ double s_kc[3];                // LeanConst source (see make_lean_const)
+  __shared__ double s_kc[4];                // LeanConst source (see make_lean_const)
   __shared__ double s_wsx[EP_MAX_THREADS / 32], s_wsy[EP_MAX_THREADS / 32];
   __shared__ unsigned long long s_wq[EP_MAX_THREADS / 32][4];
   __shared__ int s_last;
@@ -465,6 +476,7 @@ ep_kernel(const __grid_constant__ EPParams P) {
     s_kc[1] = 0.375;
     reinterpret_cast<unsigned*>(s_kc)[4] = 1u;
     reinterpret_cast<unsigned*>(s_kc)[5] = 0x200000u;
+    reinterpret_cast<unsigned*>(s_kc)[6] = 0x3FF00000u;
   }
   __syncthreads();
 
@@ -500,15 +512,15 @@ ep_kernel(const __grid_constant__ EPParams P) {
     uint64_t iters = n_t / PER_IT;
     const LeanConst K = make_lean_const(static_cast<unsigned>(__cvta_generic_to_shared(s_kc)));
     Stage<W> s0, s1;
-    if (iters) gen_stage<A32, W>(vlo, vhi, P, tab, s0);
+    if (iters) gen_stage<A32, W>(vlo, vhi, P, tab, s0, K.exp_hi);
     while (iters) {
       const unsigned ci = iters < IT_PER_CHUNK ? unsigned(iters) : IT_PER_CHUNK;
       PairAcc A{0.0, 0.0, 0u};
 #pragma unroll 1
       for (unsigned i = 0; i < ci; ++i) {
-        gen_stage<A32, W>(vlo, vhi, P, tab, s1);
+        gen_stage<A32, W>(vlo, vhi, P, tab, s1, K.exp_hi);
         transform_stage<W>(s0, P, K, A, s_rare);
-        gen_stage<A32, W>(vlo, vhi, P, tab, s0);
+        gen_stage<A32, W>(vlo, vhi, P, tab, s0, K.exp_hi);
         transform_stage<W>(s1, P, K, A, s_rare);
       }
       flush(A);
