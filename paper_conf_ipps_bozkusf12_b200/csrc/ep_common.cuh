@@ -40,8 +40,14 @@ constexpr int NJUMP = 46;
 // bits) of t' rounded to the nearest bucket centre c, inv[u] is a
 // float-exact approximation of 1/c, r = fma(t', inv[u], -1) (|r| <= 2^-9) and
 // T[u] = RN(2 ln(inv[u] / 4)), so that -2 ln t = T[u] - 2 ln(1 + r).
-constexpr int LOG_K = 8;                       // mantissa bits per exponent
-constexpr int LOG_EMIN = -16;                  // table covers t >= ~2^LOG_EMIN
+#ifndef EP_LOG_K
+#define EP_LOG_K 9
+#endif
+#ifndef EP_LOG_EMIN
+#define EP_LOG_EMIN -16
+#endif
+constexpr int LOG_K = EP_LOG_K;                // mantissa bits per exponent (8: |r| <= 2^-9, 9: 2^-10)
+constexpr int LOG_EMIN = EP_LOG_EMIN;          // table covers t >= ~2^LOG_EMIN
 constexpr int LOG_SHIFT = 20 - LOG_K;          // hi-word shift to the index
 constexpr uint32_t LOG_BIAS_TOP = 1023 - 2;    // biased exponent of t' = 1/4
 constexpr uint32_t LOG_IDX_MIN = uint32_t(int(LOG_BIAS_TOP) + LOG_EMIN) << LOG_K;

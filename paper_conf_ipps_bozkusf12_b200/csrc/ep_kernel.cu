@@ -370,7 +370,9 @@ __device__ __forceinline__ void transform_stage(const Stage<W>& S, const EPParam
     else
       acc[k] = S.t[k] <= 0.25;
     r[k] = fma(S.t[k], S.eInv[k], -1.0);
-#if EP_KMODE == 1
+#if EP_LOG_K >= 9
+    c[k] = fma(r[k], K.c6, 0.5);  // K.c6 holds c5 = -2/5 (20-bit) for the degree-5 series
+#elif EP_KMODE == 1
     c[k] = fma(r[k], EP_C6, P.coef[1]);  // c6 immediate (b slot), c5 uniform (param -> UR)
 #elif EP_KMODE == 2
     c[k] = fma(r[k], P.coef[0], EP_C5);  // c6 uniform (param -> UR, b slot), c5 immediate
@@ -378,8 +380,10 @@ __device__ __forceinline__ void transform_stage(const Stage<W>& S, const EPParam
     c[k] = fma(r[k], K.c6, EP_C5);
 #endif
   }
+#if EP_LOG_K < 9
 #pragma unroll
   for (int k = 0; k < W; ++k) c[k] = fma(c[k], r[k], 0.5);
+#endif
 #pragma unroll
   for (int k = 0; k < W; ++k) c[k] = fma(c[k], r[k], P.coef[2]);
 #pragma unroll
@@ -472,7 +476,7 @@ ep_kernel(const __grid_constant__ EPParams P) {
   }
   if (tid < 7) s_rare[tid] = 0;
   if (tid == 0) {
-    s_kc[0] = EP_C6;
+    s_kc[0] = EP_LOG_K >= 9 ? EP_C5 : EP_C6;
     s_kc[1] = 0.375;
     reinterpret_cast<unsigned*>(s_kc)[4] = 1u;
     reinterpret_cast<unsigned*>(s_kc)[5] = 0x200000u;
