@@ -39,9 +39,9 @@ PAPER_CONTEXT = {"class": "C", "mops": 3057, "hw": "Tesla C2050/C2070, OpenCL, 2
 
 # Algorithmic FP64 lane-operations per pair: 6 always
 # (2 maps, 2 squares, 1 add, 1 compare) + pi/4 * 19 for accepted pairs
-# (ln 7, sqrt(L/t) 7, X and Y 2, max 1, sums 2).
+# (ln 6, sqrt(L/t) 7, X and Y 2, max 1, sums 2) -- ln: r, 4 Horner, reconstruction (K=9 table).
 ALG_OPS_ALWAYS = 6
-ALG_OPS_ACCEPTED = 19
+ALG_OPS_ACCEPTED = 18
 P_ACCEPT = 0.7853981633974483
 ALG_OPS_PER_PAIR = ALG_OPS_ALWAYS + P_ACCEPT * ALG_OPS_ACCEPTED
 FP64_LANES_PER_SM_CLK = 64          # measured: tools/probe_fp64.cu (63.9-64.1 lane-DFMA/clk/SM)
