@@ -228,3 +228,46 @@ def test_eval_rejects_wrong_array(env):
         assert e.value.code == hpl.HPL_EINVAL
     finally:
         hpl.hpl_array_free(a)
+
+
+# ------------------------------------------------- streams / graph capture
+def test_two_streams_concurrently(env, oracle_mod):
+    """Per-(device, stream) workspaces: shards launched on two streams at once."""
+    torch, hpl = env
+    M = 22
+    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+    o1 = torch.empty(13, dtype=torch.float64, device="cuda")
+    o2 = torch.empty(13, dtype=torch.float64, device="cuda")
+    for _ in range(3):
+        hpl.hpl_ep_run_shard(M, NPB_SEED, NPB_A, 0, 2, o1.data_ptr(), s1.cuda_stream)
+        hpl.hpl_ep_run_shard(M, NPB_SEED, NPB_A, 1, 2, o2.data_ptr(), s2.cuda_stream)
+    torch.cuda.synchronize()
+    g = hpl.unpack13((o1 + o2).cpu().tolist())
+    assert_parity(g, oracle_mod.run(M, NPB_SEED, NPB_A, margin=False))
+
+
+def test_cuda_graph_replay(env, oracle_mod):
+    """The single EP launch is graph-capturable (counter self-resets) and replays exactly."""
+    torch, hpl = env
+    M = 21
+    out = torch.zeros(13, dtype=torch.float64, device="cuda")
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        hpl.hpl_ep_run_shard(M, NPB_SEED, NPB_A, 0, 1, out.data_ptr(), s.cuda_stream)  # warm workspace
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        hpl.hpl_ep_run_shard(M, NPB_SEED, NPB_A, 0, 1, out.data_ptr(), s.cuda_stream)
+    ref = oracle_mod.run(M, NPB_SEED, NPB_A, margin=False)
+    for _ in range(3):
+        out.zero_()
+        g.replay()
+        torch.cuda.synchronize()
+        assert_parity(hpl.unpack13(out.cpu().tolist()), ref)
+
+
+def test_launch_count_advances(env):
+    _, hpl = env
+    c0 = hpl.hpl_ep_launch_count()
+    hpl.hpl_ep_run(10, NPB_SEED, NPB_A)
+    assert hpl.hpl_ep_launch_count() == c0 + 1
