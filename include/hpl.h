@@ -140,6 +140,44 @@ int hpl_ep_run_range(uint64_t seed, uint64_t a, uint64_t pair_begin, uint64_t np
  * uses, copied to host_out[0..n-1].  Blocking.  n <= 2^28. */
 int hpl_lcg_states(uint64_t seed, uint64_t a, uint64_t offset, uint64_t n, uint64_t* host_out);
 
+/* ---- generic eval over an index domain ----------------
+ * The paper's eval(f).global(..).local(..)(args) for
+ * hand-written CUDA kernels registered in the library (HPL captures C++
+ * kernels at run time; here they are compiled ahead of time).
+ * A global domain has 1..3 dimensions; a local domain must have the same
+ * dimensionality and divide it in every dimension.  Each
+ * point runs one kernel instance with global id (idx, idy, idz), local id
+ * (lidx, ...) and group id (gidx, ...).  Scalars are passed
+ * by value, arrays by reference. */
+typedef enum { HPL_ARG_ARRAY = 0, HPL_ARG_F64 = 1, HPL_ARG_F32 = 2, HPL_ARG_I64 = 3, HPL_ARG_I32 = 4 } hpl_arg_kind;
+typedef struct {
+  int kind;         /* hpl_arg_kind */
+  int access;       /* arrays: hpl_access the kernel needs (0 = the kernel's declared mode) */
+  hpl_array array;  /* HPL_ARG_ARRAY */
+  double f64;       /* HPL_ARG_F64 */
+  float f32;        /* HPL_ARG_F32 */
+  int64_t i64;      /* HPL_ARG_I64 */
+  int32_t i32;      /* HPL_ARG_I32 */
+} hpl_arg;
+
+/* Evaluate registered kernel `name`.  global == NULL (or ndim == 0): the
+ * global domain is the dimensions of the first argument, which must be an
+ * array.  local == NULL or all zeros: the library chooses
+ * (PAPER.md:436-437).  Before the launch every array argument read by the
+ * kernel is made device-valid (copied only if stale); after it, every array
+ * the kernel writes becomes device-valid / host-stale (the paper's automatic
+ * transfers).  Launches on the first array argument's
+ * stream and device; asynchronous.  Errors: EINVAL (unknown kernel, argument
+ * count/kind/dtype mismatch, local not dividing global, domain too large),
+ * ESTATE (an array read by the kernel has no valid copy), ECUDA. */
+int hpl_eval(const char* name, int ndim, const int64_t* global, const int64_t* local, int nargs,
+             const hpl_arg* args);
+/* Registered kernels: count, and name/signature of kernel i (static strings).
+ * Signature: comma-separated "name:TYPE:mode" for arrays (mode r, w, rw) and
+ * "name:type" for scalars. */
+int hpl_kernel_count(int* n);
+int hpl_kernel_info(int i, const char** name, const char** signature);
+
 /* ---- tuning / introspection ------------------------------------------- */
 #define HPL_EP_LEAN 0      /* table log + rsqrt-Newton transform (default)   */
 #define HPL_EP_LIBDEVICE 1 /* CUDA libdevice log / div / sqrt, as NPB writes it */

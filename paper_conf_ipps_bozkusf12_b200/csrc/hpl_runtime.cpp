@@ -13,6 +13,7 @@
 
 #include "../../include/hpl.h"
 #include "ep_launch.h"
+#include "eval_launch.h"
 
 namespace hplep {
 
@@ -367,6 +368,168 @@ int hpl_ep_launch_shape(uint64_t npairs, int* blocks, int* threads, int* smem_by
 int hpl_ep_launch_count(uint64_t* count) {
   if (!count) return set_error(HPL_EINVAL, "count is NULL");
   *count = launch_count();
+  return HPL_OK;
+}
+
+
+// ------------------------------------------------------- generic eval (F1)
+namespace {
+struct SigArg {
+  bool array;
+  int dtype;  // arrays: hpl_dtype; scalars: hpl_arg_kind
+  int mode;   // arrays: hpl_access
+};
+
+int parse_sig(const char* sig, SigArg* out, int maxn) {
+  int n = 0;
+  const char* p = sig;
+  while (*p && n < maxn) {
+    const char* e = p;
+    while (*e && *e != ',') ++e;
+    std::string item(p, e - p);
+    size_t c1 = item.find(':');
+    size_t c2 = item.find(':', c1 + 1);
+    std::string type = item.substr(c1 + 1, c2 == std::string::npos ? std::string::npos : c2 - c1 - 1);
+    SigArg a{false, 0, 0};
+    if (c2 != std::string::npos) {  // array
+      a.array = true;
+      std::string m = item.substr(c2 + 1);
+      a.mode = m == "r" ? HPL_READ : (m == "w" ? HPL_WRITE : HPL_READWRITE);
+      a.dtype = type == "F64" ? HPL_F64 : type == "F32" ? HPL_F32 : type == "U64" ? HPL_U64
+              : type == "I64" ? HPL_I64 : type == "I32" ? HPL_I32 : HPL_U32;
+    } else {
+      a.dtype = type == "f64" ? HPL_ARG_F64 : type == "f32" ? HPL_ARG_F32 : type == "i64" ? HPL_ARG_I64
+              : HPL_ARG_I32;
+    }
+    out[n++] = a;
+    p = *e ? e + 1 : e;
+  }
+  return n;
+}
+
+int64_t pow2_divisor(int64_t v, int64_t cap) {
+  int64_t d = v & -v;
+  return d < cap ? d : cap;
+}
+}  // namespace
+
+int hpl_kernel_count(int* n) {
+  if (!n) return set_error(HPL_EINVAL, "n is NULL");
+  *n = kernel_count();
+  return HPL_OK;
+}
+
+int hpl_kernel_info(int i, const char** name, const char** signature) {
+  const KernelDesc* k = kernel_at(i);
+  if (!k) return set_error(HPL_EINVAL, "kernel index %d out of range", i);
+  if (name) *name = k->name;
+  if (signature) *signature = k->signature;
+  return HPL_OK;
+}
+
+int hpl_eval(const char* name, int ndim, const int64_t* global, const int64_t* local, int nargs,
+             const hpl_arg* args) {
+  if (!name) return set_error(HPL_EINVAL, "kernel name is NULL");
+  const KernelDesc* K = kernel_find(name);
+  if (!K) return set_error(HPL_EINVAL, "no kernel named '%s'", name);
+  SigArg sig[16];
+  const int ns = parse_sig(K->signature, sig, 16);
+  if (nargs != ns) return set_error(HPL_EINVAL, "%s takes %d arguments (%s), got %d", name, ns, K->signature, nargs);
+  if (nargs > 0 && !args) return set_error(HPL_EINVAL, "args is NULL");
+  for (int i = 0; i < nargs; ++i) {
+    if (sig[i].array) {
+      if (args[i].kind != HPL_ARG_ARRAY || !args[i].array)
+        return set_error(HPL_EINVAL, "%s argument %d must be an array", name, i);
+      if (args[i].array->t != sig[i].dtype)
+        return set_error(HPL_EINVAL, "%s argument %d has the wrong element type", name, i);
+      if (args[i].access != 0 && args[i].access != sig[i].mode)
+        return set_error(HPL_EINVAL, "%s argument %d: access mode differs from the kernel's", name, i);
+    } else if (args[i].kind != sig[i].dtype) {
+      return set_error(HPL_EINVAL, "%s argument %d must be a scalar of kind %d", name, i, sig[i].dtype);
+    }
+  }
+  // ---- global domain: given, or the first argument's dims
+  EvalDomain D;
+  D.ndim = 0;
+  for (int i = 0; i < 3; ++i) D.global[i] = D.local[i] = 1;
+  if (global == nullptr || ndim == 0) {
+    if (nargs == 0 || !sig[0].array) return set_error(HPL_EINVAL, "no global domain and no array first argument");
+    const hpl_array a0 = args[0].array;
+    if (a0->ndim < 1) return set_error(HPL_EINVAL, "the first argument is a scalar array");
+    D.ndim = a0->ndim;
+    for (int i = 0; i < D.ndim; ++i) D.global[i] = a0->dims[i];
+  } else {
+    if (ndim < 1 || ndim > 3) return set_error(HPL_EINVAL, "domains have 1..3 dimensions");
+    D.ndim = ndim;
+    for (int i = 0; i < ndim; ++i) {
+      if (global[i] <= 0) return set_error(HPL_EINVAL, "global[%d] must be > 0", i);
+      D.global[i] = global[i];
+    }
+  }
+  // ---- local domain: given (must divide the global one) or chosen
+  bool chosen = true;
+  if (local) for (int i = 0; i < D.ndim; ++i) if (local[i] != 0) chosen = false;
+  if (chosen) {
+    int64_t budget = 256;
+    for (int i = 0; i < D.ndim; ++i) {
+      D.local[i] = pow2_divisor(D.global[i], budget);
+      budget /= D.local[i];
+    }
+  } else {
+    int64_t prod = 1;
+    for (int i = 0; i < D.ndim; ++i) {
+      if (local[i] <= 0 || D.global[i] % local[i] != 0)
+        return set_error(HPL_EINVAL, "local[%d] = %lld must divide global[%d] = %lld", i, (long long)local[i], i,
+                         (long long)D.global[i]);
+      D.local[i] = local[i];
+      prod *= local[i];
+    }
+    if (prod > 1024 || D.local[2] > 64) return set_error(HPL_EINVAL, "local domain too large for one group (<= 1024 threads)");
+  }
+  if (D.global[0] / D.local[0] > 0x7FFFFFFFll || D.global[1] / D.local[1] > 65535 || D.global[2] / D.local[2] > 65535)
+    return set_error(HPL_EINVAL, "global domain too large");
+  // ---- arrays: same device, large enough, coherence before the launch
+  void* ptrs[16] = {nullptr};
+  int device = -1;
+  cudaStream_t stream = nullptr;
+  for (int i = 0; i < nargs; ++i) {
+    if (!sig[i].array) continue;
+    hpl_array a = args[i].array;
+    if (device < 0) {
+      device = a->device;
+      stream = a->stream;
+    } else if (a->device != device) {
+      return set_error(HPL_EINVAL, "array arguments live on different devices");
+    }
+    const int64_t need = K->need(D, i);
+    if (need > a->count) return set_error(HPL_EINVAL, "%s argument %d holds %lld elements, needs %lld", name, i,
+                                          (long long)a->count, (long long)need);
+  }
+  if (device < 0) {
+    int rc = current_device(&device);
+    if (rc) return rc;
+  }
+  DeviceGuard g(device);
+  if (g.rc) return g.rc;
+  for (int i = 0; i < nargs; ++i) {
+    if (!sig[i].array) continue;
+    hpl_array a = args[i].array;
+    if (sig[i].mode & HPL_READ) {
+      int rc = hpl_array_sync(a, HPL_DEVICE, HPL_READ);  // copies only if stale
+      if (rc) return rc;
+    }
+    if (a->stream != stream) {  // order this array's pending work before the launch
+      cudaError_t e = cudaStreamSynchronize(a->stream);
+      if (e != cudaSuccess) return set_cuda_error(e, "cudaStreamSynchronize");
+    }
+    ptrs[i] = a->dev;
+  }
+  int rc = K->launch(D, ptrs, args, stream);
+  if (rc) return rc;
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return set_cuda_error(e, name);
+  for (int i = 0; i < nargs; ++i)
+    if (sig[i].array && (sig[i].mode & HPL_WRITE)) args[i].array->valid = HPL_DEVICE;
   return HPL_OK;
 }
 

@@ -32,7 +32,16 @@ EXPORTS = (
     "hpl_array_info", "hpl_array_set_stream",
     "hpl_ep_eval", "hpl_ep_run", "hpl_ep_run_shard", "hpl_ep_run_range",
     "hpl_lcg_states", "hpl_ep_set_config", "hpl_ep_launch_shape", "hpl_ep_launch_count",
+    "hpl_eval", "hpl_kernel_count", "hpl_kernel_info",
 )
+HPL_ARG_ARRAY, HPL_ARG_F64, HPL_ARG_F32, HPL_ARG_I64, HPL_ARG_I32 = 0, 1, 2, 3, 4
+
+
+class HplArg(ctypes.Structure):
+    """C struct hpl_arg (include/hpl.h)."""
+    _fields_ = [("kind", ctypes.c_int), ("access", ctypes.c_int), ("array", ctypes.c_void_p),
+                ("f64", ctypes.c_double), ("f32", ctypes.c_float), ("i64", ctypes.c_int64),
+                ("i32", ctypes.c_int32)]
 
 
 class HPLError(RuntimeError):
@@ -77,6 +86,9 @@ def _load() -> ctypes.CDLL:
         "hpl_ep_set_config": (c_int, [c_int, c_int, c_int]),
         "hpl_ep_launch_shape": (c_int, [c_u64, P(c_int), P(c_int), P(c_int)]),
         "hpl_ep_launch_count": (c_int, [P(c_u64)]),
+        "hpl_eval": (c_int, [ctypes.c_char_p, c_int, P(c_i64), P(c_i64), c_int, P(HplArg)]),
+        "hpl_kernel_count": (c_int, [P(c_int)]),
+        "hpl_kernel_info": (c_int, [c_int, P(ctypes.c_char_p), P(ctypes.c_char_p)]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)
@@ -204,6 +216,53 @@ def hpl_ep_launch_count() -> int:
     c = ctypes.c_uint64()
     _check(_load().hpl_ep_launch_count(ctypes.byref(c)), "hpl_ep_launch_count")
     return c.value
+
+
+# ------------------------------------------------------- generic eval (F1)
+def _arg(v) -> HplArg:
+    a = HplArg()
+    if isinstance(v, tuple):
+        kind, val = v
+        if kind == "array":
+            a.kind, a.array = HPL_ARG_ARRAY, val
+        elif kind == "f64":
+            a.kind, a.f64 = HPL_ARG_F64, val
+        elif kind == "f32":
+            a.kind, a.f32 = HPL_ARG_F32, val
+        elif kind == "i64":
+            a.kind, a.i64 = HPL_ARG_I64, val
+        elif kind == "i32":
+            a.kind, a.i32 = HPL_ARG_I32, val
+        else:
+            raise ValueError(kind)
+    elif isinstance(v, float):
+        a.kind, a.f64 = HPL_ARG_F64, v
+    else:  # an hpl_array handle
+        a.kind, a.array = HPL_ARG_ARRAY, v
+    return a
+
+
+def hpl_eval(name: str, args, global_=None, local=None) -> None:
+    """eval(name).global(global_).local(local)(*args); arrays are handles,
+    scalars floats (f64) or (kind, value) tuples."""
+    arr = (HplArg * max(len(args), 1))(*[_arg(v) for v in args])
+    nd = len(global_) if global_ else 0
+    gl, ll = list(global_ or []), list(local or [])
+    g = (ctypes.c_int64 * max(3, len(gl)))(*(gl + [0] * (3 - len(gl))))
+    l = (ctypes.c_int64 * max(3, len(ll)))(*(ll + [0] * (3 - len(ll))))
+    _check(_load().hpl_eval(name.encode(), nd, g if nd else None, l if local else None, len(args), arr),
+           "hpl_eval")
+
+
+def hpl_kernels() -> dict:
+    n = ctypes.c_int()
+    _check(_load().hpl_kernel_count(ctypes.byref(n)), "hpl_kernel_count")
+    out = {}
+    for i in range(n.value):
+        nm, sg = ctypes.c_char_p(), ctypes.c_char_p()
+        _check(_load().hpl_kernel_info(i, ctypes.byref(nm), ctypes.byref(sg)), "hpl_kernel_info")
+        out[nm.value.decode()] = sg.value.decode()
+    return out
 
 
 def unpack13(words) -> dict:

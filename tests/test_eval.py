@@ -1,0 +1,180 @@
+"""Generic eval over index domains: the paper's own example
+kernels run through hpl_eval, checked against their plain definitions
+(numpy, IEEE roundings as the kernels write them) and the paper's Fig. 2
+statement about local ids.
+"""
+import ctypes
+
+import numpy as np
+import pytest
+
+
+@pytest.fixture(scope="module")
+def hpl():
+    from paper_conf_ipps_bozkusf12_b200 import build
+    build.build()
+    from paper_conf_ipps_bozkusf12_b200 import hpl as h
+    return h
+
+
+# ------------------------------------------------------------------- CPU
+def test_registry(hpl):
+    k = hpl.hpl_kernels()
+    assert set(k) >= {"domain_ids", "saxpy", "dotp"}
+    assert k["saxpy"] == "y:F64:rw,x:F64:r,a:f64"
+
+
+def test_bad_calls_rejected_without_gpu(hpl):
+    for name, args in [("no_such_kernel", []), ("saxpy", [1.0]), ("saxpy", [1.0, 2.0, 3.0]),
+                       ("dotp", [("array", None), ("array", None), ("array", None)])]:
+        with pytest.raises(hpl.HPLError) as e:
+            hpl.hpl_eval(name, args)
+        assert e.value.code == hpl.HPL_EINVAL
+
+
+# ------------------------------------------------------------------- GPU
+@pytest.fixture(scope="module")
+def gpu(hpl):
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    hpl.hpl_set_device(0)
+    return hpl
+
+
+def _host(hpl, a, dtype, n):
+    p = hpl.hpl_array_data(a, hpl.HPL_HOST)
+    return np.ctypeslib.as_array((ctypes.c_byte * (n * np.dtype(dtype).itemsize)).from_address(p)).view(dtype)
+
+
+@pytest.mark.gpu
+def test_fig2_domain_ids(gpu):
+    """Fig. 2: global 4x8, local 2x4; threads
+    (1,2), (1,6), (3,2), (3,6) all have local id (1,2)."""
+    hpl = gpu
+    gx, gy, lx, ly = 4, 8, 2, 4
+    a = hpl.hpl_array_alloc(hpl.HPL_I32, [gx * gy * 9])
+    try:
+        hpl.hpl_eval("domain_ids", [a], global_=[gx, gy], local=[lx, ly])
+        hpl.hpl_array_sync(a, hpl.HPL_HOST, hpl.HPL_READ)
+        ids = _host(hpl, a, np.int32, gx * gy * 9).reshape(gy, gx, 9)
+        for y in range(gy):
+            for x in range(gx):
+                i = ids[y, x]
+                assert tuple(i[0:3]) == (x, y, 0)
+                assert tuple(i[3:6]) == (x % lx, y % ly, 0)
+                assert tuple(i[6:9]) == (x // lx, y // ly, 0)
+        for (x, y) in [(1, 2), (1, 6), (3, 2), (3, 6)]:
+            assert tuple(ids[y, x, 3:5]) == (1, 2)
+    finally:
+        hpl.hpl_array_free(a)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("dims", [[1000], [96, 7], [6, 10, 4], [1 << 20]])
+def test_default_local_covers_domain_once(gpu, dims):
+    """Library-chosen local domain: every point exactly once,
+    ids consistent (g = group * local + lid)."""
+    hpl = gpu
+    n = int(np.prod(dims))
+    a = hpl.hpl_array_alloc(hpl.HPL_I32, [n * 9])
+    try:
+        hpl.hpl_eval("domain_ids", [a], global_=dims)
+        hpl.hpl_array_sync(a, hpl.HPL_HOST, hpl.HPL_READ)
+        ids = _host(hpl, a, np.int32, n * 9).reshape(n, 9)
+        d3 = list(dims) + [1] * (3 - len(dims))
+        gidx = ids[:, 0] + d3[0] * (ids[:, 1] + d3[1] * ids[:, 2])
+        assert np.array_equal(gidx, np.arange(n))
+        loc = ids[:, 3:6].max(axis=0) + 1
+        assert np.array_equal(ids[:, 0:3], ids[:, 6:9] * loc + ids[:, 3:6])
+        assert all(d % l == 0 for d, l in zip(d3, loc))
+    finally:
+        hpl.hpl_array_free(a)
+
+
+@pytest.mark.gpu
+def test_fig3_saxpy(gpu):
+    """Fig. 3: y user-owned storage, x library-owned, default
+    global domain = dims of y; y[idx] = a*x[idx] + y[idx] (two roundings)."""
+    hpl = gpu
+    rng = np.random.default_rng(3)
+    n = 1000
+    myvector = rng.standard_normal(n)
+    y0 = myvector.copy()
+    x = hpl.hpl_array_alloc(hpl.HPL_F64, [n])
+    y = hpl.hpl_array_alloc(hpl.HPL_F64, [n], myvector.ctypes.data)
+    try:
+        xh = _host(hpl, x, np.float64, n)
+        xh[:] = rng.standard_normal(n)
+        hpl.hpl_array_sync(x, hpl.HPL_HOST, hpl.HPL_WRITE)  # host copy written
+        a = 2.5
+        hpl.hpl_eval("saxpy", [y, x, a])
+        assert hpl.hpl_array_info(y)["valid"] == hpl.HPL_DEVICE
+        assert np.array_equal(myvector, y0)  # host copy untouched until synced
+        hpl.hpl_array_sync(y, hpl.HPL_HOST, hpl.HPL_READ)
+        assert np.array_equal(myvector, a * xh + y0)
+        # a second eval reuses the still-valid device copy of x: a host edit
+        # not announced with a WRITE sync is (by contract) not uploaded
+        x_old, y1 = xh.copy(), myvector.copy()
+        xh[:] = 0.0
+        hpl.hpl_eval("saxpy", [y, x, a])
+        hpl.hpl_array_sync(y, hpl.HPL_HOST, hpl.HPL_READ)
+        assert np.array_equal(myvector, a * x_old + y1)
+        # announcing the edit makes the next eval upload it
+        hpl.hpl_array_sync(x, hpl.HPL_HOST, hpl.HPL_WRITE)
+        y2 = myvector.copy()
+        hpl.hpl_eval("saxpy", [y, x, a])
+        hpl.hpl_array_sync(y, hpl.HPL_HOST, hpl.HPL_READ)
+        assert np.array_equal(myvector, y2)
+    finally:
+        hpl.hpl_array_free(x)
+        hpl.hpl_array_free(y)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("N,M", [(256, 32), (4096, 128), (1 << 20, 256)])
+def test_fig4_dotp(gpu, N, M):
+    """Fig. 4: per-group partial dot products through Local
+    memory, lane 0 sums in order into pSums[gidx]; host sums nGroup partials."""
+    hpl = gpu
+    rng = np.random.default_rng(N)
+    ng = N // M
+    v1 = hpl.hpl_array_alloc(hpl.HPL_F32, [N])
+    v2 = hpl.hpl_array_alloc(hpl.HPL_F32, [N])
+    ps = hpl.hpl_array_alloc(hpl.HPL_F32, [ng])
+    try:
+        a1, a2, p = _host(hpl, v1, np.float32, N), _host(hpl, v2, np.float32, N), _host(hpl, ps, np.float32, ng)
+        a1[:] = rng.standard_normal(N).astype(np.float32)
+        a2[:] = rng.standard_normal(N).astype(np.float32)
+        p[:] = 0
+        for h in (v1, v2, ps):
+            hpl.hpl_array_sync(h, hpl.HPL_HOST, hpl.HPL_WRITE)
+        hpl.hpl_eval("dotp", [v1, v2, ps], global_=[N], local=[M])
+        hpl.hpl_array_sync(ps, hpl.HPL_HOST, hpl.HPL_READ)
+        prods = (a1 * a2).astype(np.float32).reshape(ng, M)
+        want = np.zeros(ng, dtype=np.float32)
+        for i in range(M):  # lane 0's sequential float32 sum
+            want = (want + prods[:, i]).astype(np.float32)
+        assert np.array_equal(p, want)
+        dot = float(np.sum(p.astype(np.float64)))
+        assert abs(dot - float(np.dot(a1.astype(np.float64), a2.astype(np.float64)))) < 1e-3 * N ** 0.5
+    finally:
+        for h in (v1, v2, ps):
+            hpl.hpl_array_free(h)
+
+
+@pytest.mark.gpu
+def test_eval_domain_errors(gpu):
+    hpl = gpu
+    a = hpl.hpl_array_alloc(hpl.HPL_I32, [4 * 8 * 9])
+    b = hpl.hpl_array_alloc(hpl.HPL_F32, [16])
+    try:
+        for g, l in [([4, 8], [3, 4]), ([4, 8], [2, 5]), ([4, 8, 1, 1], None), ([8, 8], [2, 4])]:
+            with pytest.raises(hpl.HPLError) as e:
+                hpl.hpl_eval("domain_ids", [a], global_=g, local=l)
+            assert e.value.code == hpl.HPL_EINVAL
+        with pytest.raises(hpl.HPLError):  # wrong dtype for saxpy
+            hpl.hpl_eval("saxpy", [b, b, 1.0])
+    finally:
+        hpl.hpl_array_free(a)
+        hpl.hpl_array_free(b)
