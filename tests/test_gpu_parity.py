@@ -271,3 +271,18 @@ def test_launch_count_advances(env):
     c0 = hpl.hpl_ep_launch_count()
     hpl.hpl_ep_run(10, NPB_SEED, NPB_A)
     assert hpl.hpl_ep_launch_count() == c0 + 1
+
+
+def test_npb_class_E_verification_sums(env):
+    """Class E (M = 40, 2^41 uniforms, ~2 s on one B200): no oracle run is
+    affordable, so the pin is NPB's published verification sums (1e-8) plus
+    the statistical invariants."""
+    _, hpl = env
+    M, sxr, syr = npb_verify()["E"]
+    assert M == 40
+    sx, sy, q = hpl.hpl_ep_run(M, NPB_SEED, NPB_A)
+    assert abs((sx - sxr) / sxr) <= 1e-8 and abs((sy - syr) / syr) <= 1e-8
+    n, p = 2 ** M, math.pi / 4
+    gc = sum(q)
+    assert abs(gc - n * p) < 5 * math.sqrt(n * p * (1 - p))
+    assert q[9] == 0 and q[8] <= 2
