@@ -140,6 +140,15 @@ int hpl_ep_run_range(uint64_t seed, uint64_t a, uint64_t pair_begin, uint64_t np
  * uses, copied to host_out[0..n-1].  Blocking.  n <= 2^28. */
 int hpl_lcg_states(uint64_t seed, uint64_t a, uint64_t offset, uint64_t n, uint64_t* host_out);
 
+/* ---- reduction -----------------------------------------
+ * The paper's fifth benchmark, "the addition of 16M single-precision floating
+ * point values" (SHOC): *dev_out =
+ * sum(dev_in[0..n-1]) accumulated in FP64 (deterministic order), written as
+ * one double into device memory, asynchronously on `stream`.  dev_in needs
+ * only 4-byte alignment; n may be 0 (result 0).  Also registered for
+ * hpl_eval as "sum_f32" (in:F32:r, out:F64:w). */
+int hpl_reduce_sum_f32(const float* dev_in, int64_t n, double* dev_out, void* stream);
+
 /* ---- generic eval over an index domain ----------------
  * The paper's eval(f).global(..).local(..)(args) for
  * hand-written CUDA kernels registered in the library (HPL captures C++

@@ -8,12 +8,15 @@
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
+#include <mutex>
 #include <new>
+#include <vector>
 #include <string>
 
 #include "../../include/hpl.h"
 #include "ep_launch.h"
 #include "eval_launch.h"
+#include "reduce_launch.h"
 
 namespace hplep {
 
@@ -531,6 +534,55 @@ int hpl_eval(const char* name, int ndim, const int64_t* global, const int64_t* l
   for (int i = 0; i < nargs; ++i)
     if (sig[i].array && (sig[i].mode & HPL_WRITE)) args[i].array->valid = HPL_DEVICE;
   return HPL_OK;
+}
+
+
+// ------------------------------------------------------------ reduction (F2)
+namespace {
+struct RedWs {
+  int device;
+  cudaStream_t stream;
+  hplep::ReduceWorkspace ws;
+  int sms;
+};
+std::mutex g_red_mu;
+std::vector<RedWs> g_red;
+
+int reduce_workspace(int device, cudaStream_t stream, hplep::ReduceWorkspace** ws, int* sms) {
+  std::lock_guard<std::mutex> lk(g_red_mu);
+  for (auto& w : g_red)
+    if (w.device == device && w.stream == stream) {
+      *ws = &w.ws;
+      *sms = w.sms;
+      return 0;
+    }
+  RedWs w{device, stream, {}, 0};
+  cudaError_t e = cudaDeviceGetAttribute(&w.sms, cudaDevAttrMultiProcessorCount, device);
+  if (e != cudaSuccess) return set_cuda_error(e, "cudaDeviceGetAttribute");
+  w.ws.capacity = w.sms * 4;
+  e = cudaMalloc(&w.ws.partials, sizeof(double) * w.ws.capacity);
+  if (e == cudaSuccess) e = cudaMalloc(&w.ws.counter, sizeof(unsigned));
+  if (e == cudaSuccess) e = cudaMemset(w.ws.counter, 0, sizeof(unsigned));
+  if (e != cudaSuccess) return set_cuda_error(e, "reduce workspace");
+  g_red.push_back(w);
+  *ws = &g_red.back().ws;
+  *sms = w.sms;
+  return 0;
+}
+}  // namespace
+
+int hpl_reduce_sum_f32(const float* dev_in, int64_t n, double* dev_out, void* stream) {
+  if (n < 0) return set_error(HPL_EINVAL, "n must be >= 0");
+  if (!dev_out || (n > 0 && !dev_in)) return set_error(HPL_EINVAL, "NULL pointer");
+  if (reinterpret_cast<uintptr_t>(dev_in) & 3) return set_error(HPL_EINVAL, "dev_in must be 4-byte aligned");
+  int dev;
+  int rc = current_device(&dev);
+  if (rc) return rc;
+  hplep::ReduceWorkspace* ws;
+  int sms;
+  rc = reduce_workspace(dev, static_cast<cudaStream_t>(stream), &ws, &sms);
+  if (rc) return rc;
+  return hplep::launch_reduce_sum_f32(dev_in, n, dev_out, *ws, sms, static_cast<cudaStream_t>(stream));
 }
 
 }  // extern "C"

@@ -32,7 +32,7 @@ EXPORTS = (
     "hpl_array_info", "hpl_array_set_stream",
     "hpl_ep_eval", "hpl_ep_run", "hpl_ep_run_shard", "hpl_ep_run_range",
     "hpl_lcg_states", "hpl_ep_set_config", "hpl_ep_launch_shape", "hpl_ep_launch_count",
-    "hpl_eval", "hpl_kernel_count", "hpl_kernel_info",
+    "hpl_eval", "hpl_kernel_count", "hpl_kernel_info", "hpl_reduce_sum_f32",
 )
 HPL_ARG_ARRAY, HPL_ARG_F64, HPL_ARG_F32, HPL_ARG_I64, HPL_ARG_I32 = 0, 1, 2, 3, 4
 
@@ -88,6 +88,7 @@ def _load() -> ctypes.CDLL:
         "hpl_ep_launch_count": (c_int, [P(c_u64)]),
         "hpl_eval": (c_int, [ctypes.c_char_p, c_int, P(c_i64), P(c_i64), c_int, P(HplArg)]),
         "hpl_kernel_count": (c_int, [P(c_int)]),
+        "hpl_reduce_sum_f32": (c_int, [c_void_p, c_i64, c_void_p, c_void_p]),
         "hpl_kernel_info": (c_int, [c_int, P(ctypes.c_char_p), P(ctypes.c_char_p)]),
     }
     for name, (res, args) in sig.items():
@@ -216,6 +217,11 @@ def hpl_ep_launch_count() -> int:
     c = ctypes.c_uint64()
     _check(_load().hpl_ep_launch_count(ctypes.byref(c)), "hpl_ep_launch_count")
     return c.value
+
+
+# ---------------------------------------------------------- reduction (F2)
+def hpl_reduce_sum_f32(dev_in: int, n: int, dev_out: int, stream: int | None = None) -> None:
+    _check(_load().hpl_reduce_sum_f32(dev_in, n, dev_out, stream or None), "hpl_reduce_sum_f32")
 
 
 # ------------------------------------------------------- generic eval (F1)

@@ -1,0 +1,41 @@
+"""F2 measurement: hpl_reduce_sum_f32 GB/s vs the measured HBM copy peak.
+
+python tools/bench_reduce.py [--n N ...]   (one JSON line per size)
+Inputs are resident in HBM; L2 (126 MB) is flushed by a 256 MB write between
+timed launches; CUDA events on the launching stream.  Algorithmic bytes =
+4 n (each float read once; the 8-byte result and ~5 KB of partials ignored).
+"""
+import argparse, json, os, sys
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch
+from paper_conf_ipps_bozkusf12_b200 import hpl
+
+ap = argparse.ArgumentParser()
+ap.add_argument("--n", type=int, nargs="*", default=[16 << 20, 256 << 20])
+ap.add_argument("--iters", type=int, default=10)
+a = ap.parse_args()
+root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+pk = json.load(open(os.path.join(root, "MEASURED_PEAKS.json"))) if os.path.exists(os.path.join(root, "MEASURED_PEAKS.json")) else {}
+peak = float(pk.get("hbm_gbs", 6650.0))
+torch.cuda.set_device(0); hpl.hpl_set_device(0)
+s = torch.cuda.current_stream()
+flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+for n in a.n:
+    x = torch.randn(n, dtype=torch.float32, device="cuda")
+    out = torch.empty(1, dtype=torch.float64, device="cuda")
+    for _ in range(3):
+        hpl.hpl_reduce_sum_f32(x.data_ptr(), n, out.data_ptr(), s.cuda_stream)
+    ts = []
+    for _ in range(a.iters):
+        flush.zero_()
+        e0 = torch.cuda.Event(enable_timing=True); e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(s)
+        hpl.hpl_reduce_sum_f32(x.data_ptr(), n, out.data_ptr(), s.cuda_stream)
+        e1.record(s); e1.synchronize()
+        ts.append(e0.elapsed_time(e1) / 1e3)
+    t = sorted(ts)[len(ts) // 2]
+    gbs = 4 * n / t / 1e9
+    print(json.dumps({"workload": "sum of %d f32 (F2)" % n, "median_s": t, "GB/s": round(gbs, 1),
+                      "roofline": {"bound": "hbm", "achieved": round(gbs, 1), "peak": peak, "unit": "GB/s",
+                                   "frac": round(gbs / peak, 4), "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy)"},
+                      "result": out.item(), "torch_sum_f64": float(x.double().sum())}), flush=True)
