@@ -37,3 +37,26 @@ def uniforms(M: int) -> int:
 
 def pairs(M: int) -> int:
     return 1 << M
+
+
+# ---------------------------------------------------------------- F4: spmv
+# Fig. 7's spmv size: "a 16K x 16K matrix with a 1% of non zeros"
+# (PAPER.md:950-951); Fig. 5's toy: nRows 1024, M = 8.
+SPMV_ROWS = 16 * 1024
+SPMV_DENSITY = 0.01
+
+
+def make_csr(n_rows, n_cols, density, seed):
+    """Seeded synthetic CSR matrix (numpy): each row gets Binomial(n_cols,
+    density) distinct uniformly random sorted columns, values U(-1, 1) float32.
+    Returns rowptr (int32, n_rows+1), cols (int32), A (float32)."""
+    import numpy as np
+    rng = np.random.default_rng(seed)
+    counts = rng.binomial(n_cols, density, n_rows)
+    rowptr = np.zeros(n_rows + 1, dtype=np.int64)
+    np.cumsum(counts, out=rowptr[1:])
+    cols = np.empty(int(rowptr[-1]), dtype=np.int32)
+    for i in range(n_rows):
+        cols[rowptr[i]:rowptr[i + 1]] = np.sort(rng.choice(n_cols, counts[i], replace=False))
+    A = rng.uniform(-1.0, 1.0, int(rowptr[-1])).astype(np.float32)
+    return rowptr.astype(np.int32), cols, A
