@@ -320,6 +320,9 @@ __device__ __forceinline__ void lean_pairs(unsigned& vlo, unsigned& vhi, const E
   }
 }
 
+#ifndef EP_T2MODE
+#define EP_T2MODE 1    // 1: t2 = g + g (e cc) instead of g + (g e) cc
+#endif
 #ifndef EP_KMODE
 #define EP_KMODE 0     // 1: loop constants as immediates + kernel-parameter (uniform) operands
 #endif
@@ -406,6 +409,8 @@ __device__ __forceinline__ void transform_stage(const Stage<W>& S, const EPParam
     t2[k] = fma(__dmul_rn(g[k], e[k]), fma(e[k], 0.375, P.coef[4]), g[k]);
 #elif EP_KMODE == 2
     t2[k] = fma(__dmul_rn(g[k], e[k]), fma(e[k], P.coef[3], 0.5), g[k]);
+#elif EP_T2MODE == 1
+    t2[k] = fma(g[k], __dmul_rn(e[k], fma(e[k], K.c0375, 0.5)), g[k]);  // g (1 + e cc)
 #else
     t2[k] = fma(__dmul_rn(g[k], e[k]), fma(e[k], K.c0375, 0.5), g[k]);
 #endif
