@@ -320,6 +320,14 @@ __device__ __forceinline__ void lean_pairs(unsigned& vlo, unsigned& vhi, const E
   }
 }
 
+#ifndef EP_TMA_TABLE
+#define EP_TMA_TABLE 0 // 1: load the log table with cp.async.bulk (TMA) + mbarrier: ~2 us
+                       // less per launch, but ptxas then allocates the hot loop's registers
+                       // slightly worse (+0.8 operand reads/pair, -1.5 % at class D)
+#endif
+#ifndef EP_TMA_WAIT_LATE
+#define EP_TMA_WAIT_LATE 0  // 1: wait for the table after the skip-ahead instead of before
+#endif
 #ifndef EP_T2MODE
 #define EP_T2MODE 1    // 1: t2 = g + g (e cc) instead of g + (g e) cc
 #endif
@@ -470,14 +478,34 @@ ep_kernel(const __grid_constant__ EPParams P) {
   __shared__ unsigned long long s_wq[EP_MAX_THREADS / 32][4];
   __shared__ int s_last;
   __shared__ double s_fin[13];
+  __shared__ long long s_fold[EP_MAX_THREADS / 16][13];
 
   const unsigned tid = threadIdx.x;
   unsigned tab;  // opaque copy: keeps the shared base in a register (no per-use rematerialisation)
   asm volatile("mov.u32 %0, %1;" : "=r"(tab) : "r"(static_cast<unsigned>(__cvta_generic_to_shared(smem_raw))));
-  if (VARIANT == HPL_VARIANT_LEAN) {
+  // Table -> shared memory with TMA bulk copies (cp.async.bulk, one thread,
+  // completion counted on an mbarrier): one 131-KB stream at L2 bandwidth
+  // instead of 16 dependent load/store rounds per thread (~8 us per launch).
+  __shared__ __align__(8) unsigned long long s_mbar;
+  const unsigned mbar = static_cast<unsigned>(__cvta_generic_to_shared(&s_mbar));
+  if (VARIANT == HPL_VARIANT_LEAN && !EP_TMA_TABLE) {
     const double2* src = reinterpret_cast<const double2*>(P.table);
     double2* dst = reinterpret_cast<double2*>(smem_raw);
     for (unsigned i = tid; i < LOG_TAB; i += blockDim.x) dst[i] = __ldg(src + i);
+  }
+  if (VARIANT == HPL_VARIANT_LEAN && EP_TMA_TABLE && tid == 0) {
+    constexpr unsigned BYTES = LOG_TAB * sizeof(LogEntry), CHUNK = 32768;
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(mbar));
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("{\n\t.reg .b64 st;\n\tmbarrier.arrive.expect_tx.shared::cta.b64 st, [%0], %1;\n\t}"
+                 ::"r"(mbar), "r"(BYTES) : "memory");
+    const unsigned dst = static_cast<unsigned>(__cvta_generic_to_shared(smem_raw));
+    const char* src = reinterpret_cast<const char*>(P.table);
+    for (unsigned off = 0; off < BYTES; off += CHUNK) {
+      const unsigned n = BYTES - off < CHUNK ? BYTES - off : CHUNK;
+      asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                   ::"r"(dst + off), "l"(src + off), "r"(n), "r"(mbar) : "memory");
+    }
   }
   if (tid < 7) s_rare[tid] = 0;
   if (tid == 0) {
@@ -487,7 +515,15 @@ ep_kernel(const __grid_constant__ EPParams P) {
     reinterpret_cast<unsigned*>(s_kc)[5] = 0x200000u;
     reinterpret_cast<unsigned*>(s_kc)[6] = 0x3FF00000u;
   }
-  __syncthreads();
+  __syncthreads();  // mbarrier initialised before anyone waits on it
+#if !EP_TMA_WAIT_LATE
+  if (VARIANT == HPL_VARIANT_LEAN && EP_TMA_TABLE) {
+    unsigned done = 0;
+    while (!done)
+      asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], 0;\n\t"
+                   "selp.u32 %0, 1, 0, p;\n\t}" : "=r"(done) : "r"(mbar) : "memory");
+  }
+#endif
 
   // ---- A2: this thread's pair range and start state
   const uint64_t gid = uint64_t(blockIdx.x) * blockDim.x + tid;
@@ -495,6 +531,15 @@ ep_kernel(const __grid_constant__ EPParams P) {
   const uint64_t p0 = gid * P.base + (gid < P.extra ? gid : P.extra);
   const uint64_t v0 = state_to_v(jump_state(P.x_begin, 2 * p0, P.jump));
   unsigned vlo = unsigned(v0), vhi = unsigned(v0 >> 32);
+#if EP_TMA_WAIT_LATE
+  // the skip-ahead above overlapped the table's bulk copy; wait for it now
+  if (VARIANT == HPL_VARIANT_LEAN && EP_TMA_TABLE) {
+    unsigned done = 0;
+    while (!done)
+      asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], 0;\n\t"
+                   "selp.u32 %0, 1, 0, p;\n\t}" : "=r"(done) : "r"(mbar) : "memory");
+  }
+#endif
 
   double sx = 0.0, sy = 0.0;
   unsigned q0 = 0, q1 = 0, q2 = 0, q3 = 0;
@@ -606,19 +651,34 @@ ep_kernel(const __grid_constant__ EPParams P) {
   }
   __syncthreads();
   if (!s_last) return;
-  // last block: word w of the result summed over blocks 0..G-1 in order
+  // last block: 16-thread groups; thread (group gi, word w) folds word w of
+  // partials gi, gi + ng, ... (independent loads in flight), then thread w
+  // folds the groups in order — fixed order, so bitwise deterministic.
   __threadfence();
-  if (tid < 13) {
-    const unsigned G = gridDim.x;
-    if (tid < 2) {
-      double s = 0.0;
-      for (unsigned b = 0; b < G; ++b) s += __ldcg(tid == 0 ? &P.partials[b].sx : &P.partials[b].sy);
-      s_fin[tid] = s;
-    } else {
-      unsigned long long s = 0;
-      for (unsigned b = 0; b < G; ++b)
-        s += __ldcg(tid < 12 ? &P.partials[b].q[tid - 2] : &P.partials[b].big);
-      s_fin[tid] = static_cast<double>(s);  // exact: < 2^53
+  {
+    const unsigned G = gridDim.x, ng = blockDim.x >> 4, gi = tid >> 4, w = tid & 15;
+    if (w < 13) {
+      if (w < 2) {
+        double sacc = 0.0;
+        for (unsigned b = gi; b < G; b += ng) sacc += __ldcg(w == 0 ? &P.partials[b].sx : &P.partials[b].sy);
+        s_fold[gi][w] = __double_as_longlong(sacc);
+      } else {
+        unsigned long long sacc = 0;
+        for (unsigned b = gi; b < G; b += ng) sacc += __ldcg(w < 12 ? &P.partials[b].q[w - 2] : &P.partials[b].big);
+        s_fold[gi][w] = static_cast<long long>(sacc);
+      }
+    }
+    __syncthreads();
+    if (tid < 13) {
+      if (tid < 2) {
+        double sacc = 0.0;
+        for (unsigned g = 0; g < ng; ++g) sacc += __longlong_as_double(s_fold[g][tid]);
+        s_fin[tid] = sacc;
+      } else {
+        unsigned long long sacc = 0;
+        for (unsigned g = 0; g < ng; ++g) sacc += static_cast<unsigned long long>(s_fold[g][tid]);
+        s_fin[tid] = static_cast<double>(sacc);  // exact: < 2^53
+      }
     }
   }
   __syncthreads();
@@ -809,11 +869,25 @@ int launch_shape(int device, uint64_t npairs, const EPConfig& cfg, int* blocks, 
   const int sm_bytes = cfg.variant == HPL_VARIANT_LEAN ? int(LOG_TAB * sizeof(LogEntry)) : 0;
   int bps = cfg.blocks_per_sm;
   if (bps <= 0) {
-    int occ = 0;
-    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, pick_kernel(cfg.variant, true, thr),
-                                                                  thr, sm_bytes);
-    if (e != cudaSuccess) return set_cuda_error(e, "cudaOccupancyMaxActiveBlocksPerMultiprocessor");
-    bps = occ > 0 ? occ : 1;
+    // occupancy per (device, variant, block size), cached: the query costs
+    // microseconds of host time that would sit inside small launches
+    static std::mutex occ_mu;
+    static std::vector<long long> occ_cache;  // key << 8 | occupancy
+    const long long key = (static_cast<long long>(device) << 20) | (static_cast<long long>(cfg.variant) << 12) | thr;
+    {
+      std::lock_guard<std::mutex> lk(occ_mu);
+      for (long long v : occ_cache)
+        if ((v >> 8) == key) bps = int(v & 0xFF);
+    }
+    if (bps <= 0) {
+      int occ = 0;
+      cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, pick_kernel(cfg.variant, true, thr),
+                                                                    thr, sm_bytes);
+      if (e != cudaSuccess) return set_cuda_error(e, "cudaOccupancyMaxActiveBlocksPerMultiprocessor");
+      bps = occ > 0 ? occ : 1;
+      std::lock_guard<std::mutex> lk(occ_mu);
+      occ_cache.push_back((key << 8) | bps);
+    }
   }
   // at least EP_MIN_PAIRS_PER_THREAD pairs per thread so skip-ahead stays negligible
   uint64_t want = (npairs + uint64_t(thr) * EP_MIN_PAIRS_PER_THREAD - 1) / (uint64_t(thr) * EP_MIN_PAIRS_PER_THREAD);
