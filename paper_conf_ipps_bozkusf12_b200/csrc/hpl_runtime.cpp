@@ -306,8 +306,12 @@ int hpl_ep_eval(int M, uint64_t seed, uint64_t a, int rank, int nranks, hpl_arra
 
 int hpl_ep_run(int M, uint64_t seed, uint64_t a, double* sx, double* sy, uint64_t q[10]) {
   if (!sx || !sy || !q) return set_error(HPL_EINVAL, "NULL output pointer");
+  uint64_t b0, n0;
+  int rc = shard_range(M, 0, 1, &b0, &n0);  // argument errors before any CUDA call
+  if (!rc) rc = validate(seed, a);
+  if (rc) return rc;
   int dev;
-  int rc = current_device(&dev);
+  rc = current_device(&dev);
   if (rc) return rc;
   // one cached 13-word Array per thread and device (the paper's Array with
   // a library-owned host copy)
