@@ -320,6 +320,9 @@ __device__ __forceinline__ void lean_pairs(unsigned& vlo, unsigned& vhi, const E
   }
 }
 
+#ifndef EP_PIPE_ORDER
+#define EP_PIPE_ORDER 0  // 1: single stage, transform then generate (no ping-pong)
+#endif
 #ifndef EP_TMA_TABLE
 #define EP_TMA_TABLE 0 // 1: load the log table with cp.async.bulk (TMA) + mbarrier: ~2 us
                        // less per launch, but ptxas then allocates the hot loop's registers
@@ -555,7 +558,7 @@ ep_kernel(const __grid_constant__ EPParams P) {
     // 8-bit packed counters overflow after 255 pairs: <= 252 pairs per flush.
     // Tail pairs first, so the pipelined loop's one-group overshoot past the
     // thread's range is never transformed.
-    constexpr unsigned PER_IT = 2 * W, IT_PER_CHUNK = 252 / PER_IT;
+    constexpr unsigned PER_IT = (EP_PIPE_ORDER == 1 ? 1 : 2) * W, IT_PER_CHUNK = 252 / PER_IT;
     const unsigned tail = unsigned(n_t % PER_IT);
     if (tail) {
       PairAcc A{0.0, 0.0, 0u};
@@ -572,10 +575,16 @@ ep_kernel(const __grid_constant__ EPParams P) {
       PairAcc A{0.0, 0.0, 0u};
 #pragma unroll 1
       for (unsigned i = 0; i < ci; ++i) {
+#if EP_PIPE_ORDER == 1
+        transform_stage<W>(s0, P, K, A, s_rare);
+        gen_stage<A32, W>(vlo, vhi, P, tab, s0, K.exp_hi);
+        (void)s1;
+#else
         gen_stage<A32, W>(vlo, vhi, P, tab, s1, K.exp_hi);
         transform_stage<W>(s0, P, K, A, s_rare);
         gen_stage<A32, W>(vlo, vhi, P, tab, s0, K.exp_hi);
         transform_stage<W>(s1, P, K, A, s_rare);
+#endif
       }
       flush(A);
       iters -= ci;
