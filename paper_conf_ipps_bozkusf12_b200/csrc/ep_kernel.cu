@@ -320,6 +320,10 @@ __device__ __forceinline__ void lean_pairs(unsigned& vlo, unsigned& vhi, const E
   }
 }
 
+#ifndef EP_LOOP_UNROLL
+#define EP_LOOP_UNROLL 1  // unroll of the pipelined group loop (codegen/register-allocation knob)
+#endif
+constexpr int kLoopUnroll = EP_LOOP_UNROLL;  // (#pragma arguments are not macro-expanded)
 #ifndef EP_PIPE_ORDER
 #define EP_PIPE_ORDER 0  // 1: single stage, transform then generate (no ping-pong)
 #endif
@@ -573,7 +577,7 @@ ep_kernel(const __grid_constant__ EPParams P) {
     while (iters) {
       const unsigned ci = iters < IT_PER_CHUNK ? unsigned(iters) : IT_PER_CHUNK;
       PairAcc A{0.0, 0.0, 0u};
-#pragma unroll 1
+#pragma unroll kLoopUnroll
       for (unsigned i = 0; i < ci; ++i) {
 #if EP_PIPE_ORDER == 1
         transform_stage<W>(s0, P, K, A, s_rare);
