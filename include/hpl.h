@@ -187,6 +187,12 @@ int hpl_eval(const char* name, int ndim, const int64_t* global, const int64_t* l
 int hpl_kernel_count(int* n);
 int hpl_kernel_info(int i, const char** name, const char** signature);
 
+/* Test hook: pairs [pair_begin, pair_begin + n) through the production lean
+ * transform code (gen_stage / transform_stage), one pair per thread; writes
+ * host_out[4i..4i+3] = {t, X, Y, l} with l = -1 for pairs taken by the rare
+ * path (X, Y still filled) and -2 for rejected pairs.  Blocking; n <= 2^26. */
+int hpl_ep_pairs_debug(uint64_t seed, uint64_t a, uint64_t pair_begin, uint64_t n, double* host_out);
+
 /* ---- tuning / introspection ------------------------------------------- */
 #define HPL_EP_LEAN 0      /* table log + rsqrt-Newton transform (default)   */
 #define HPL_EP_LIBDEVICE 1 /* CUDA libdevice log / div / sqrt, as NPB writes it */

@@ -375,9 +375,10 @@ __device__ __forceinline__ void gen_stage(unsigned& vlo, unsigned& vhi, const EP
     asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(S.eT[k]), "=d"(S.eInv[k]) : "r"((S.u[k] << 4) + tab));
 }
 
-template <int W>
+template <int W, bool DBG = false>
 __device__ __forceinline__ void transform_stage(const Stage<W>& S, const EPParams& P, const LeanConst& K,
-                                                PairAcc& A, unsigned long long* s_rare) {
+                                                PairAcc& A, unsigned long long* s_rare,
+                                                double* dbg = nullptr) {
   double r[W], c[W], L[W], p[W], y0[W], e[W], g[W], t2[W], X[W], Y[W];
   unsigned l[W];
   bool acc[W], ok[W];
@@ -440,6 +441,12 @@ __device__ __forceinline__ void transform_stage(const Stage<W>& S, const EPParam
       A.cnt += bin_increment(l[k], K.one);
     }
     any_rare |= acc[k] && !ok[k];
+    if (DBG) {  // test hook (hpl_ep_pairs_debug): t, X, Y, l (-1 rare path, -2 rejected)
+      dbg[4 * k + 0] = 4.0 * S.t[k];
+      dbg[4 * k + 1] = ok[k] ? X[k] : 0.0;
+      dbg[4 * k + 2] = ok[k] ? Y[k] : 0.0;
+      dbg[4 * k + 3] = ok[k] ? double(l[k]) : (acc[k] ? -1.0 : -2.0);
+    }
   }
   if (any_rare) {
 #pragma unroll
@@ -449,8 +456,43 @@ __device__ __forceinline__ void transform_stage(const Stage<W>& S, const EPParam
         A.csx += o.dx;
         A.csy += o.dy;
         A.cnt += o.dcnt;
+        if (DBG) {
+          dbg[4 * k + 1] = o.dx;
+          dbg[4 * k + 2] = o.dy;
+        }
       }
   }
+}
+
+// Test hook: every pair of [pair_begin, pair_begin + n) through the production
+// gen_stage / transform_stage code (one pair per thread), writing t, X, Y, l.
+template <bool A32>
+__global__ void __launch_bounds__(256) ep_pairs_debug_kernel(const __grid_constant__ EPParams P, uint64_t n,
+                                                             double* out) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  __shared__ unsigned long long s_rare[7];
+  __shared__ double s_kc[4];
+  for (unsigned i = threadIdx.x; i < LOG_TAB; i += blockDim.x)
+    reinterpret_cast<double2*>(smem_raw)[i] = __ldg(reinterpret_cast<const double2*>(P.table) + i);
+  if (threadIdx.x < 7) s_rare[threadIdx.x] = 0;
+  if (threadIdx.x == 0) {
+    s_kc[0] = EP_LOG_K >= 9 ? EP_C5 : EP_C6;
+    s_kc[1] = 0.375;
+    reinterpret_cast<unsigned*>(s_kc)[4] = 1u;
+    reinterpret_cast<unsigned*>(s_kc)[5] = 0x200000u;
+    reinterpret_cast<unsigned*>(s_kc)[6] = 0x3FF00000u;
+  }
+  __syncthreads();
+  const uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  const unsigned tab = static_cast<unsigned>(__cvta_generic_to_shared(smem_raw));
+  const LeanConst K = make_lean_const(static_cast<unsigned>(__cvta_generic_to_shared(s_kc)));
+  const uint64_t v0 = state_to_v(jump_state(P.x_begin, 2 * i, P.jump));
+  unsigned vlo = unsigned(v0), vhi = unsigned(v0 >> 32);
+  Stage<1> S;
+  gen_stage<A32, 1>(vlo, vhi, P, tab, S, K.exp_hi);
+  PairAcc A{0.0, 0.0, 0u};
+  transform_stage<1, true>(S, P, K, A, s_rare, out + 4 * i);
 }
 
 // NPB's own formulation with CUDA libdevice log / div / sqrt (A/B variant).
@@ -766,6 +808,26 @@ uint64_t host_jump(uint64_t x, uint64_t k, const uint64_t* J) {
   return x;
 }
 
+// Kernel parameters shared by every EP launch: jump table J[i] = a^(2^i),
+// multiplier words, a^(k+1) table, constants, and the range's start state
+// x_begin = seed * a^(2 pair_begin) mod 2^46.
+static void init_params(EPParams& P, uint64_t seed, uint64_t a, uint64_t pair_begin) {
+  std::memset(&P, 0, sizeof(P));
+  build_jump_table(a, P.jump);
+  P.a = a;
+  P.a_lo = unsigned(a);
+  P.a_hi = unsigned(a >> 32);
+  uint64_t ak = a & MASK46;
+  for (int k = 0; k < 8; ++k) {  // a^(k+1) mod 2^46
+    P.apow_lo[k] = unsigned(ak);
+    P.apow_hi[k] = unsigned(ak >> 32);
+    ak = mulmod46(ak, a);
+  }
+  const double coef[6] = {EP_C6, EP_C5, -2.0 / 3.0, 0.375, 0.5, 0x1p-200};
+  for (int i = 0; i < 6; ++i) P.coef[i] = coef[i];
+  P.x_begin = host_jump(seed & MASK46, 2 * pair_begin, P.jump);
+}
+
 // Lean-log table, built in 80-bit long double on the host.
 void build_log_table(std::vector<LogEntry>& tab) {
   tab.resize(LOG_TAB);
@@ -928,22 +990,7 @@ int launch_ep(int device, uint64_t seed, uint64_t a, uint64_t pair_begin, uint64
   if (rc) return rc;
 
   EPParams P;
-  std::memset(&P, 0, sizeof(P));
-  build_jump_table(a, P.jump);
-  P.a = a;
-  P.a_lo = unsigned(a);
-  P.a_hi = unsigned(a >> 32);
-  {
-    uint64_t ak = a & MASK46;
-    for (int k = 0; k < 8; ++k) {  // a^(k+1) mod 2^46
-      P.apow_lo[k] = unsigned(ak);
-      P.apow_hi[k] = unsigned(ak >> 32);
-      ak = mulmod46(ak, a);
-    }
-  }
-  const double coef[6] = {EP_C6, EP_C5, -2.0 / 3.0, 0.375, 0.5, 0x1p-200};
-  for (int i = 0; i < 6; ++i) P.coef[i] = coef[i];
-  P.x_begin = host_jump(seed & MASK46, 2 * pair_begin, P.jump);
+  init_params(P, seed, a, pair_begin);
   P.npairs = npairs;
   const uint64_t T = uint64_t(blocks) * threads;
   P.base = npairs / T;
@@ -967,6 +1014,28 @@ int launch_ep(int device, uint64_t seed, uint64_t a, uint64_t pair_begin, uint64
 unsigned long long launch_count() {
   std::lock_guard<std::mutex> lk(g_mu);
   return g_launches;
+}
+
+int launch_pairs_debug(int device, uint64_t seed, uint64_t a, uint64_t pair_begin, uint64_t n,
+                       double* dev_out, cudaStream_t stream) {
+  const LogEntry* tab;
+  int sms;
+  int rc = device_state(device, &tab, &sms);
+  if (rc) return rc;
+  EPParams P;
+  init_params(P, seed, a, pair_begin);
+  P.table = tab;
+  const int smem = int(LOG_TAB * sizeof(LogEntry));
+  const bool a32 = (a >> 32) == 0;
+  auto k = a32 ? ep_pairs_debug_kernel<true> : ep_pairs_debug_kernel<false>;
+  cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e != cudaSuccess) return set_cuda_error(e, "cudaFuncSetAttribute(debug)");
+  const uint64_t blocks = (n + 255) / 256;
+  if (blocks == 0) return 0;
+  k<<<unsigned(blocks), 256, smem, stream>>>(P, n, dev_out);
+  e = cudaGetLastError();
+  if (e != cudaSuccess) return set_cuda_error(e, "ep_pairs_debug_kernel launch");
+  return 0;
 }
 
 int launch_lcg_states(uint64_t seed, uint64_t a, uint64_t offset, uint64_t n, uint64_t* dev_out,

@@ -589,4 +589,26 @@ int hpl_reduce_sum_f32(const float* dev_in, int64_t n, double* dev_out, void* st
   return hplep::launch_reduce_sum_f32(dev_in, n, dev_out, *ws, sms, static_cast<cudaStream_t>(stream));
 }
 
+
+int hpl_ep_pairs_debug(uint64_t seed, uint64_t a, uint64_t pair_begin, uint64_t n, double* host_out) {
+  int rc = validate(seed, a);
+  if (rc) return rc;
+  if (n > (uint64_t(1) << 26)) return set_error(HPL_EINVAL, "n must be <= 2^26");
+  if (n == 0) return HPL_OK;
+  if (!host_out) return set_error(HPL_EINVAL, "host_out is NULL");
+  int dev;
+  rc = current_device(&dev);
+  if (rc) return rc;
+  double* d = nullptr;
+  cudaError_t e = cudaMalloc(&d, n * 4 * sizeof(double));
+  if (e != cudaSuccess) return set_cuda_error(e, "cudaMalloc(debug)");
+  rc = launch_pairs_debug(dev, seed, a, pair_begin, n, d, nullptr);
+  if (!rc) {
+    e = cudaMemcpy(host_out, d, n * 4 * sizeof(double), cudaMemcpyDeviceToHost);
+    if (e != cudaSuccess) rc = set_cuda_error(e, "cudaMemcpy(debug)");
+  }
+  cudaFree(d);
+  return rc;
+}
+
 }  // extern "C"

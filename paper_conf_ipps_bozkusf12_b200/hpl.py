@@ -33,6 +33,7 @@ EXPORTS = (
     "hpl_ep_eval", "hpl_ep_run", "hpl_ep_run_shard", "hpl_ep_run_range",
     "hpl_lcg_states", "hpl_ep_set_config", "hpl_ep_launch_shape", "hpl_ep_launch_count",
     "hpl_eval", "hpl_kernel_count", "hpl_kernel_info", "hpl_reduce_sum_f32",
+    "hpl_ep_pairs_debug",
 )
 HPL_ARG_ARRAY, HPL_ARG_F64, HPL_ARG_F32, HPL_ARG_I64, HPL_ARG_I32 = 0, 1, 2, 3, 4
 
@@ -89,6 +90,7 @@ def _load() -> ctypes.CDLL:
         "hpl_eval": (c_int, [ctypes.c_char_p, c_int, P(c_i64), P(c_i64), c_int, P(HplArg)]),
         "hpl_kernel_count": (c_int, [P(c_int)]),
         "hpl_reduce_sum_f32": (c_int, [c_void_p, c_i64, c_void_p, c_void_p]),
+        "hpl_ep_pairs_debug": (c_int, [c_u64, c_u64, c_u64, c_u64, P(c_double)]),
         "hpl_kernel_info": (c_int, [c_int, P(ctypes.c_char_p), P(ctypes.c_char_p)]),
     }
     for name, (res, args) in sig.items():
@@ -199,6 +201,13 @@ def hpl_lcg_states(seed: int, a: int, offset: int, n: int) -> list[int]:
     buf = (ctypes.c_uint64 * max(n, 1))()
     _check(_load().hpl_lcg_states(seed, a, offset, n, buf), "hpl_lcg_states")
     return list(buf[:n])
+
+
+def hpl_ep_pairs_debug(seed: int, a: int, pair_begin: int, n: int):
+    """Per-pair (t, X, Y, l) from the production transform code (test hook)."""
+    buf = (ctypes.c_double * max(4 * n, 1))()
+    _check(_load().hpl_ep_pairs_debug(seed, a, pair_begin, n, buf), "hpl_ep_pairs_debug")
+    return buf
 
 
 def hpl_ep_set_config(variant: int = HPL_EP_LEAN, threads_per_block: int = 0,
