@@ -286,3 +286,18 @@ def test_npb_class_E_verification_sums(env):
     gc = sum(q)
     assert abs(gc - n * p) < 5 * math.sqrt(n * p * (1 - p))
     assert q[9] == 0 and q[8] <= 2
+
+
+@pytest.mark.parametrize("case", range(8))
+def test_random_streams(env, oracle_mod, case):
+    """Seeded random (seed, a, range) combinations incl. wide multipliers and
+    ranges near the 2^43-pair limit, vs the oracle."""
+    rng = random.Random(1000 + case)
+    seed = rng.randrange(1 << 46)
+    if seed == 1 << 45:
+        seed += 1
+    a = (rng.randrange(1 << 46) | 1) if case % 2 else (rng.randrange(1 << 31) | 1)
+    n = rng.randrange(1, 1 << 21)
+    begin = rng.randrange((1 << 43) - n)
+    g = gpu_range(env, seed, a, begin, n)
+    assert_parity(g, oracle_mod.run_pairs(seed, a, begin, n))
