@@ -198,3 +198,20 @@ def test_statistics_class_S(oracle_mod):
     chi2 = sum((r.q[l] - r.gc * probs[l]) ** 2 / (r.gc * probs[l]) for l in range(6))
     assert chi2 < 25  # 5 dof; P(chi2 > 25) ~ 1e-4
     assert abs(r.sx) < 5 * math.sqrt(r.gc) and abs(r.sy) < 5 * math.sqrt(r.gc)
+
+
+def test_stored_large_class_goldens_match_npb():
+    """tests/golden/oracle_ep.json (written by oracle/ only) against NPB's
+    published verification sums for B, C, D and the recalled class-B counts."""
+    from _golden import oracle_golden
+    g = oracle_golden()
+    ver = npb_verify()
+    for cls in ("B", "C", "D"):
+        assert cls in g, cls
+        M, sxr, syr = ver[cls]
+        assert g[cls]["M"] == M and g[cls]["npairs"] == 2 ** M and g[cls]["qbig"] == 0
+        assert abs((g[cls]["sx"] - sxr) / sxr) <= 1e-10 and abs((g[cls]["sy"] - syr) / syr) <= 1e-10
+        assert sum(g[cls]["q"]) == g[cls]["gc"]
+        assert g[cls]["min_margin_ulp"] > 8
+    M, gc, q = npb_counts()["B"]
+    assert g["B"]["gc"] == gc and g["B"]["q"] == q
