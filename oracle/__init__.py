@@ -68,6 +68,8 @@ def _load():
         R = ctypes.POINTER(_Result)
         lib.ep_oracle_randlc.argtypes = [ctypes.POINTER(d), d]
         lib.ep_oracle_randlc.restype = d
+        lib.ep_oracle_pair_t.argtypes = [d, d]
+        lib.ep_oracle_pair_t.restype = d
         lib.ep_oracle_states.argtypes = [d, d, u64, u64, ctypes.POINTER(u64)]
         lib.ep_oracle_states.restype = i
         lib.ep_oracle_an.argtypes = [d, i]
@@ -93,6 +95,11 @@ def randlc(x: float, a: float) -> tuple[float, float]:
     xx = ctypes.c_double(x)
     u = _load().ep_oracle_randlc(ctypes.byref(xx), a)
     return u, xx.value
+
+
+def pair_t(x1: float, x2: float) -> float:
+    """t = x1**2 + x2**2 exactly as the oracle's Gaussian loop evaluates it."""
+    return _load().ep_oracle_pair_t(x1, x2)
 
 
 def states(seed: int, a: int, offset: int, n: int) -> list[int]:

@@ -215,3 +215,25 @@ def test_stored_large_class_goldens_match_npb():
         assert g[cls]["min_margin_ulp"] > 8
     M, gc, q = npb_counts()["B"]
     assert g["B"]["gc"] == gc and g["B"]["q"] == q
+
+
+def _rn(dec):
+    return float(dec)  # Decimal -> nearest double (correct rounding)
+
+
+def test_t_is_unfused(oracle_mod):
+    """R5 pin: t = RN(RN(x1²) + RN(x2²)), not the fused RN(x1² + RN(x2²)).
+    Searches LCG-shaped inputs (x = 2u-1, u = k 2^-46) where the two differ and
+    checks the oracle returns the unfused value there (and everywhere)."""
+    rng = random.Random(55)
+    differ = 0
+    with localcontext() as ctx:
+        ctx.prec = 60
+        for _ in range(20000):
+            x1 = 2.0 * (rng.randrange(MOD46) * 2.0 ** -46) - 1.0
+            x2 = 2.0 * (rng.randrange(MOD46) * 2.0 ** -46) - 1.0
+            unfused = x1 * x1 + x2 * x2                     # Python floats never fuse
+            fused = _rn(Decimal(x1) * Decimal(x1) + Decimal(x2 * x2))
+            assert oracle_mod.pair_t(x1, x2) == unfused
+            differ += fused != unfused
+    assert differ > 1000  # the check is discriminating
