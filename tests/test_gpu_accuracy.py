@@ -75,3 +75,15 @@ def test_exact_boundary_t_equals_one(hpl):
     out = np.frombuffer(hpl.hpl_ep_pairs_debug(NPB_SEED, NPB_A, 777, n), dtype=np.float64).reshape(n, 4)
     one = out[:, 0] == 1.0
     assert np.all(out[one, 1] == 0.0) and np.all(out[one, 3] == 0.0)
+
+
+def test_worked_example_first_pairs(hpl):
+    """P4 on the GPU: the production transform reproduces the first six pairs."""
+    import os
+    path = os.path.join(os.path.dirname(os.path.abspath(__file__)), "golden", "ep_first_pairs.txt")
+    rows = [l.split() for l in open(path) if l.strip() and not l.startswith("#")]
+    out = np.frombuffer(hpl.hpl_ep_pairs_debug(NPB_SEED, NPB_A, 0, len(rows)), dtype=np.float64).reshape(-1, 4)
+    for r, o in zip(rows, out):
+        X, Y = float(r[1]), float(r[2])
+        assert abs(o[1] - X) <= 4 * np.spacing(abs(X)) and abs(o[2] - Y) <= 4 * np.spacing(abs(Y))
+        assert int(o[3]) == int(r[3])

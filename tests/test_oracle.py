@@ -237,3 +237,27 @@ def test_t_is_unfused(oracle_mod):
             assert oracle_mod.pair_t(x1, x2) == unfused
             differ += fused != unfused
     assert differ > 1000  # the check is discriminating
+
+
+def test_worked_example_first_pairs():
+    """P4: the first six pairs (tests/golden/ep_first_pairs.txt) re-derived from
+    exact-integer LCG states and 50-digit decimal arithmetic."""
+    import os
+    path = os.path.join(os.path.dirname(os.path.abspath(__file__)), "golden", "ep_first_pairs.txt")
+    rows = [l.split() for l in open(path) if l.strip() and not l.startswith("#")]
+    x = NPB_SEED
+    with localcontext() as ctx:
+        ctx.prec = 50
+        for r in rows:
+            x = NPB_A * x % MOD46
+            u1 = x
+            x = NPB_A * x % MOD46
+            u2 = x
+            x1 = 2.0 * (u1 * 2.0 ** -46) - 1.0
+            x2 = 2.0 * (u2 * 2.0 ** -46) - 1.0
+            t = x1 * x1 + x2 * x2
+            assert t <= 1.0
+            f = (Decimal(-2) * Decimal(t).ln() / Decimal(t)).sqrt()
+            X, Y = float(Decimal(x1) * f), float(Decimal(x2) * f)
+            assert abs(X - float(r[1])) <= 4 * math.ulp(X) and abs(Y - float(r[2])) <= 4 * math.ulp(Y)
+            assert int(max(abs(X), abs(Y))) == int(r[3])
