@@ -55,10 +55,15 @@ constexpr uint32_t LOG_IDX_MAX = uint32_t(LOG_BIAS_TOP) << LOG_K;  // bucket of 
 constexpr uint32_t LOG_N = LOG_IDX_MAX - LOG_IDX_MIN + 1;  // 4097 real entries
 // u = (hi(t') + LOG_ADD) >> LOG_SHIFT  (mod 2^32), valid iff u < LOG_N
 constexpr uint32_t LOG_ADD = (uint32_t(1) << (LOG_SHIFT - 1)) - (LOG_IDX_MIN << LOG_SHIFT);
-// Entry LOG_N is a sentinel {T = 2^1000, inv = 0}: every t' outside the table
-// (rejected t' > ~1/4, or t < 2^LOG_EMIN) is clamped onto it, which makes
-// t2 ~ 2^500 and hence l >= 4, routing the pair to the exact rare path.
-constexpr uint32_t LOG_TAB = LOG_N + 1;
+// Entries LOG_N .. LOG_N + 511 are reject sentinels {T = 2^1000, inv = 0}: they
+// cover every rejected t' in (~1/4, 1/2) and make t2 ~ 2^500, so X, Y are huge
+// (l >= 4 and, in the FP32 binning, a selector >= 2^21).  Entry LOG_TINY =
+// LOG_N + 512 is the sentinel for t' below the table (the index wraps around
+// and is clamped onto it): {T = 60, inv = 0} gives L ~ 64.6 and hence
+// max(|X|,|Y|) in [5.6, 8.1], routing the pair to the exact rare path.
+// (The older acceptance mode clamps at LOG_N, whose entry is a reject sentinel.)
+constexpr uint32_t LOG_TINY = LOG_N + 512;
+constexpr uint32_t LOG_TAB = LOG_TINY + 1;
 
 struct LogEntry {
   double T;    // RN(2 ln(inv / 4))

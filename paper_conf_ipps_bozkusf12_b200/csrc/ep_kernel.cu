@@ -54,14 +54,34 @@ __device__ __forceinline__ unsigned bin_increment(unsigned l, unsigned one = 1u)
 }
 
 #ifndef EP_BIN_MODE
-#define EP_BIN_MODE 0  // 0: two F2I; 1: hi-word max + one F2I; 2: hi-word max + integer shift (no XU)
+#define EP_BIN_MODE 3  // 0: two F2I; 1: hi-word max + one F2I; 2: hi-word max + integer shift; 3: FP32 view of the high words (no XU)
 #endif
 // l = trunc(max(|X|,|Y|)) for the common case, and ge4 = (max(|X|,|Y|) >= 4).
 // Modes 1/2 take the max on the high words: (hi << 1) drops the sign and
 // keeps the magnitude order, and for values < 2^20 the integer part depends
 // on the high word only, so no rounding question arises.  Mode 2 then
 // truncates with integer ops: (1.f) 2^21 >> (21 - e), e = exponent.
+//
+// Mode 3 (no XU instructions): the high word h of a double with value M read
+// as an FP32 number is f(h), a monotone piecewise-linear map with f(1) = 1.875,
+// f(2) = 2, f(3) = 2.125, f(4) = 2.25 (bits 0x3FF00000, 0x40000000,
+// 0x40080000, 0x40100000).  The integer thresholds have zero low words, so
+// trunc(M) < 5 is decided exactly by h.  m = max(|f(hX)|, |f(hY)|, 1.75)
+// (one FMNMX3), then v = RM(m + 2^20 - 1.75) lands on the 1/8 grid of
+// [2^20, 2^21): bits(v) = bits(2^20) + trunc(8 (m - 1.75)) = bits(2^20) + l for
+// M < 4, and >= bits(2^20) + 4 iff M >= 4.  The returned selector is bits(v)
+// (PRMT reads its two low bits).
 __device__ __forceinline__ unsigned bin_index(double X, double Y, bool& ge4, unsigned implicit_bit) {
+  if (EP_BIN_MODE == 3) {
+    const float fx = __int_as_float(__double2hiint(X)), fy = __int_as_float(__double2hiint(Y));
+    float m;  // max(|fx|, |fy|, 1.75), NaN if either is NaN (FMNMX3.NAN)
+    asm("max.NaN.f32 %0, %1, %2, 0f3FE00000;" : "=f"(m) : "f"(fabsf(fx)), "f"(fabsf(fy)));
+    float v;
+    asm("add.rm.f32 %0, %1, 0f497FFFE4;" : "=f"(v) : "f"(m));  // 2^20 - 1.75
+    const unsigned b = __float_as_uint(v);
+    ge4 = b >= 0x49800004u;
+    return b;
+  }
   if (EP_BIN_MODE == 0) {
     const unsigned l = max(__double2uint_rz(fabs(X)), __double2uint_rz(fabs(Y)));
     ge4 = l >= 4;
@@ -140,6 +160,7 @@ struct RareOut {
 };
 __device__ __noinline__ RareOut rare_pair(double t, double x1, double x2, double X, double Y,
                                           unsigned u, unsigned long long* s_rare) {
+  if (t > 0.25) return RareOut{0.0, 0.0, 0u};  // rejected (never routed here by the fast path)
   if (u >= LOG_N) {  // t below the table: NPB's formula, libdevice log/sqrt, on
     // the unscaled t = 4 t', x = 2 x' (exact)
     const double tt = 4.0 * t;
@@ -341,6 +362,21 @@ constexpr int kLoopUnroll = EP_LOOP_UNROLL;  // (#pragma arguments are not macro
 #ifndef EP_KMODE
 #define EP_KMODE 0     // 1: loop constants as immediates + kernel-parameter (uniform) operands
 #endif
+#ifndef EP_ABL
+#define EP_ABL 0       // ablation bit set for timing studies only (results are wrong if != 0)
+#endif
+#ifndef EP_MAXSQ
+#define EP_MAXSQ 0     // 1: bin from RN(max|x'| t2) (one DMUL), sums by DFMA (needs EP_BIN_MODE 3)
+#endif
+#ifndef EP_PRED_MODE
+#define EP_PRED_MODE 0 // 1: acceptance and rare routing from the FP32 bin selector (needs EP_BIN_MODE 3)
+#endif
+#if EP_PRED_MODE == 1 && EP_BIN_MODE != 3
+#error "EP_PRED_MODE 1 needs EP_BIN_MODE 3"
+#endif
+#ifndef EP_RARE_VOTE
+#define EP_RARE_VOTE 1 // 1: rare-path branch on a warp vote (needs warp-uniform trip counts)
+#endif
 #ifndef EP_PIPE
 #define EP_PIPE 1      // 1: software-pipeline generation of group g+1 under the transform of group g
 #endif
@@ -352,6 +388,7 @@ constexpr int kLoopUnroll = EP_LOOP_UNROLL;  // (#pragma arguments are not macro
 template <int W>
 struct Stage {
   double x1[W], x2[W], t[W], eT[W], eInv[W];
+  double xm[W];  // EP_MAXSQ: the x' of larger magnitude
   unsigned u[W];
 };
 
@@ -360,19 +397,40 @@ __device__ __forceinline__ void gen_stage(unsigned& vlo, unsigned& vhi, const EP
                                           Stage<W>& S, unsigned exp_hi) {
 #pragma unroll
   for (int k = 0; k < W; ++k) {
+#if EP_ABL & 2  // ablation (timing only, wrong results): LCG step -> one add
+    vlo += P.a_lo;
+#else
     lcg_step_k<A32>(vlo, vhi, P.a_lo, P.a_hi, exp_hi);
+#endif
     S.x1[k] = __dadd_rn(__hiloint2double(int(vhi), int(vlo)), -1.5);
+#if EP_ABL & 2
+    vhi ^= vlo;
+#else
     lcg_step_k<A32>(vlo, vhi, P.a_lo, P.a_hi, exp_hi);
+#endif
     S.x2[k] = __dadd_rn(__hiloint2double(int(vhi), int(vlo)), -1.5);
   }
 #pragma unroll
   for (int k = 0; k < W; ++k) {
+#if EP_MAXSQ
+    const double s1 = __dmul_rn(S.x1[k], S.x1[k]), s2 = __dmul_rn(S.x2[k], S.x2[k]);
+    S.t[k] = __dadd_rn(s1, s2);
+    S.xm[k] = __double_as_longlong(s1) >= __double_as_longlong(s2) ? S.x1[k] : S.x2[k];
+#else
     S.t[k] = __dadd_rn(__dmul_rn(S.x1[k], S.x1[k]), __dmul_rn(S.x2[k], S.x2[k]));
-    S.u[k] = min((static_cast<unsigned>(__double2hiint(S.t[k])) + LOG_ADD) >> LOG_SHIFT, LOG_N);
+#endif
+    S.u[k] = min((static_cast<unsigned>(__double2hiint(S.t[k])) + LOG_ADD) >> LOG_SHIFT,
+                 EP_PRED_MODE == 1 ? LOG_TINY : LOG_N);
   }
 #pragma unroll
-  for (int k = 0; k < W; ++k)
+  for (int k = 0; k < W; ++k) {
+#if EP_ABL & 1  // ablation: no table lookup / index
+    S.eT[k] = S.x1[k];
+    S.eInv[k] = S.x2[k];
+#else
     asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(S.eT[k]), "=d"(S.eInv[k]) : "r"((S.u[k] << 4) + tab));
+#endif
+  }
 }
 
 template <int W, bool DBG = false>
@@ -384,7 +442,9 @@ __device__ __forceinline__ void transform_stage(const Stage<W>& S, const EPParam
   bool acc[W], ok[W];
 #pragma unroll
   for (int k = 0; k < W; ++k) {
-    if (EP_ACC_INT)
+    if (EP_PRED_MODE == 1 && !DBG)
+      acc[k] = true;  // decided by the selector below (rejects -> NaN or >= 2^21)
+    else if (EP_ACC_INT)
       acc[k] = static_cast<unsigned long long>(__double_as_longlong(S.t[k])) <= 0x3FD0000000000000ull;
     else
       acc[k] = S.t[k] <= 0.25;
@@ -413,11 +473,17 @@ __device__ __forceinline__ void transform_stage(const Stage<W>& S, const EPParam
   for (int k = 0; k < W; ++k) {
     L[k] = fma(c[k], r[k], S.eT[k]);
     p[k] = fma(L[k], S.t[k], 0x1p-200);
+#if EP_ABL & 4  // ablation: no MUFU
+    y0[k] = S.t[k];
+#else
     y0[k] = rsqrt_approx(p[k]);
+#endif
   }
 #pragma unroll
   for (int k = 0; k < W; ++k) e[k] = fma(-__dmul_rn(p[k], y0[k]), y0[k], 1.0);
   bool any_rare = false;
+  unsigned sel_min = 0xFFFFFFFFu;
+  (void)sel_min;
 #pragma unroll
   for (int k = 0; k < W; ++k) {
     g[k] = __dmul_rn(L[k], y0[k]);
@@ -425,33 +491,79 @@ __device__ __forceinline__ void transform_stage(const Stage<W>& S, const EPParam
     t2[k] = fma(__dmul_rn(g[k], e[k]), fma(e[k], 0.375, P.coef[4]), g[k]);
 #elif EP_KMODE == 2
     t2[k] = fma(__dmul_rn(g[k], e[k]), fma(e[k], P.coef[3], 0.5), g[k]);
+#elif EP_T2MODE == 2
+    t2[k] = __dmul_rn(g[k], fma(e[k], fma(e[k], K.c0375, 0.5), 1.0));  // g RN(1 + e cc): no 3-register DFMA
 #elif EP_T2MODE == 1
     t2[k] = fma(g[k], __dmul_rn(e[k], fma(e[k], K.c0375, 0.5)), g[k]);  // g (1 + e cc)
 #else
     t2[k] = fma(__dmul_rn(g[k], e[k]), fma(e[k], K.c0375, 0.5), g[k]);
 #endif
+#if EP_MAXSQ
+    // max(|X|,|Y|) = RN(|xm| t2) with xm chosen by the rounded squares (equal
+    // squares can pick the smaller |x'|: <= 1 ulp, inside reading R7's margin)
+    const double Mv = __dmul_rn(S.xm[k], t2[k]);
+    X[k] = Mv;  // placeholders: the rare path / debug hook recompute X, Y
+    Y[k] = Mv;
+#else
     X[k] = __dmul_rn(S.x1[k], t2[k]);
     Y[k] = __dmul_rn(S.x2[k], t2[k]);
+#endif
     bool ge4;
+#if EP_ABL & 8  // ablation: no binning (F2I, max, compare)
+    l[k] = 0; ge4 = false;
+#else
     l[k] = bin_index(X[k], Y[k], ge4, K.implicit_bit);
+#endif
+#if EP_ABL & 16  // ablation: no acceptance / rare predicates
+    ok[k] = true; acc[k] = true;
+#else
     ok[k] = acc[k] && !ge4;
+#endif
+#if EP_PRED_MODE == 1
+    // selector bits: < 2^20 + 4/8 ok; [.., 2^21) rare (l >= 4 or tiny t');
+    // >= 2^21 or NaN: rejected (reject sentinel, or t' > 1/4 in the 1/4 bucket,
+    // where L < 0 makes X, Y NaN and FMNMX3.NAN propagates it)
+    sel_min = min(sel_min, l[k] - 0x49800004u);
+#endif
     if (ok[k]) {
+#if EP_MAXSQ
+      A.csx = fma(S.x1[k], t2[k], A.csx);
+      A.csy = fma(S.x2[k], t2[k], A.csy);
+#else
       A.csx = __dadd_rn(A.csx, X[k]);
       A.csy = __dadd_rn(A.csy, Y[k]);
+#endif
       A.cnt += bin_increment(l[k], K.one);
     }
+#if EP_PRED_MODE != 1
     any_rare |= acc[k] && !ok[k];
+#endif
+    if (DBG && EP_MAXSQ) {
+      X[k] = __dmul_rn(S.x1[k], t2[k]);
+      Y[k] = __dmul_rn(S.x2[k], t2[k]);
+    }
     if (DBG) {  // test hook (hpl_ep_pairs_debug): t, X, Y, l (-1 rare path, -2 rejected)
       dbg[4 * k + 0] = 4.0 * S.t[k];
       dbg[4 * k + 1] = ok[k] ? X[k] : 0.0;
       dbg[4 * k + 2] = ok[k] ? Y[k] : 0.0;
-      dbg[4 * k + 3] = ok[k] ? double(l[k]) : (acc[k] ? -1.0 : -2.0);
+      dbg[4 * k + 3] = ok[k] ? double(EP_BIN_MODE == 3 ? l[k] & 3u : l[k]) : (acc[k] ? -1.0 : -2.0);
     }
   }
+#if EP_PRED_MODE == 1
+  any_rare = sel_min < 0x007FFFFCu;
+#endif
+#if EP_RARE_VOTE
+  if (DBG ? any_rare : __any_sync(0xFFFFFFFFu, any_rare)) {  // warp-uniform: no reconvergence barrier
+#else
   if (any_rare) {
+#endif
 #pragma unroll
     for (int k = 0; k < W; ++k)
-      if (acc[k] && !ok[k]) {
+      if (EP_PRED_MODE == 1 ? (l[k] - 0x49800004u < 0x007FFFFCu) : (acc[k] && !ok[k])) {
+        if (EP_MAXSQ) {
+          X[k] = __dmul_rn(S.x1[k], t2[k]);
+          Y[k] = __dmul_rn(S.x2[k], t2[k]);
+        }
         const RareOut o = rare_pair(S.t[k], S.x1[k], S.x2[k], X[k], Y[k], S.u[k], s_rare);
         A.csx += o.dx;
         A.csy += o.dy;
@@ -605,14 +717,17 @@ ep_kernel(const __grid_constant__ EPParams P) {
     // Tail pairs first, so the pipelined loop's one-group overshoot past the
     // thread's range is never transformed.
     constexpr unsigned PER_IT = (EP_PIPE_ORDER == 1 ? 1 : 2) * W, IT_PER_CHUNK = 252 / PER_IT;
-    const unsigned tail = unsigned(n_t % PER_IT);
+    // Warp-uniform trip count: every thread runs base / PER_IT pipelined
+    // iterations (base = the grid-wide floor), the rest (< PER_IT + 1 pairs)
+    // goes through the tail loop.
+    const unsigned tail = unsigned(n_t - (P.base / PER_IT) * PER_IT);
     if (tail) {
       PairAcc A{0.0, 0.0, 0u};
 #pragma unroll 1
       for (unsigned i = 0; i < tail; ++i) lean_pair<A32>(vlo, vhi, P, tab, A, s_rare);
       flush(A);
     }
-    uint64_t iters = n_t / PER_IT;
+    uint64_t iters = P.base / PER_IT;
     const LeanConst K = make_lean_const(static_cast<unsigned>(__cvta_generic_to_shared(s_kc)));
     Stage<W> s0, s1;
     if (iters) gen_stage<A32, W>(vlo, vhi, P, tab, s0, K.exp_hi);
@@ -638,7 +753,7 @@ ep_kernel(const __grid_constant__ EPParams P) {
   } else {
     // 8-bit packed counters overflow after 255 pairs: chunks of 252 = 63 x 4
     constexpr unsigned UNROLL = 4, CHUNK = 63 * UNROLL;
-    static_assert(UNROLL % W == 0, "W must divide UNROLL");
+    static_assert(EP_PIPE || UNROLL % W == 0, "W must divide UNROLL");
     uint64_t rem = n_t;
     for (; rem >= CHUNK; rem -= CHUNK) {
       PairAcc A{0.0, 0.0, 0u};
@@ -646,7 +761,7 @@ ep_kernel(const __grid_constant__ EPParams P) {
       for (unsigned i = 0; i < CHUNK / UNROLL; ++i) {
         if (VARIANT == HPL_VARIANT_LEAN) {
   #pragma unroll
-          for (unsigned j = 0; j < UNROLL / W; ++j) lean_pairs<A32, W>(vlo, vhi, P, tab, A, s_rare);
+          for (unsigned j = 0; j < UNROLL / W; ++j) lean_pairs<A32, (UNROLL % W ? 1 : W)>(vlo, vhi, P, tab, A, s_rare);
         } else {
   #pragma unroll
           for (unsigned j = 0; j < UNROLL; ++j) libdevice_pair<A32>(vlo, vhi, P, tab, A, s_rare);
@@ -778,7 +893,7 @@ static EPKernel tier_kernel(int thr) {
 #define EP_T384_W EP_ILP
 #endif
 #ifndef EP_T512_W
-#define EP_T512_W EP_ILP
+#define EP_T512_W 3  // 124 registers, no spills; +2 % over W = 2
 #endif
   if (thr <= 128) return ep_kernel<V, A32, 128, 4, 1>;   // 128 regs
   if (thr <= 256) return ep_kernel<V, A32, 256, EP_T256_MINB, EP_T256_W>;   //  85 regs (3 blocks/SM)
@@ -839,8 +954,12 @@ void build_log_table(std::vector<LogEntry>& tab) {
     tab[u].inv = (double)inv;
     tab[u].T = (double)(2.0L * logl((long double)inv * 0.25L));  // -2 ln(4 t') at r = 0
   }
-  tab[LOG_N].T = 0x1p1000;  // sentinel: forces l >= 4 -> exact rare path
-  tab[LOG_N].inv = 0.0;
+  for (uint32_t u = LOG_N; u < LOG_TINY; ++u) {  // reject sentinels (ep_common.cuh)
+    tab[u].T = 0x1p1000;
+    tab[u].inv = 0.0;
+  }
+  tab[LOG_TINY].T = 60.0;  // t' below the table -> moderate X, Y -> exact rare path
+  tab[LOG_TINY].inv = 0.0;
 }
 
 namespace {
