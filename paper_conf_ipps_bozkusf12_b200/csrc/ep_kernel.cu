@@ -158,9 +158,12 @@ struct RareOut {
   double dx, dy;
   unsigned dcnt;
 };
+// `u` is the caller's table index of t' (>= LOG_N below the table); with
+// u = ~0u the index is recomputed here (the stage then need not keep it live).
 __device__ __noinline__ RareOut rare_pair(double t, double x1, double x2, double X, double Y,
                                           unsigned u, unsigned long long* s_rare) {
   if (t > 0.25) return RareOut{0.0, 0.0, 0u};  // rejected (never routed here by the fast path)
+  if (u == ~0u) u = (static_cast<unsigned>(__double2hiint(t)) + LOG_ADD) >> LOG_SHIFT;  // wraps below the table
   if (u >= LOG_N) {  // t below the table: NPB's formula, libdevice log/sqrt, on
     // the unscaled t = 4 t', x = 2 x' (exact)
     const double tt = 4.0 * t;
@@ -365,6 +368,9 @@ constexpr int kLoopUnroll = EP_LOOP_UNROLL;  // (#pragma arguments are not macro
 #ifndef EP_ABL
 #define EP_ABL 0       // ablation bit set for timing studies only (results are wrong if != 0)
 #endif
+#ifndef EP_STAGE_U
+#define EP_STAGE_U 1   // 1: the stage keeps the table index for the rare path (register-allocation knob)
+#endif
 #ifndef EP_MAXSQ
 #define EP_MAXSQ 0     // 1: bin from RN(max|x'| t2) (one DMUL), sums by DFMA (needs EP_BIN_MODE 3)
 #endif
@@ -564,7 +570,7 @@ __device__ __forceinline__ void transform_stage(const Stage<W>& S, const EPParam
           X[k] = __dmul_rn(S.x1[k], t2[k]);
           Y[k] = __dmul_rn(S.x2[k], t2[k]);
         }
-        const RareOut o = rare_pair(S.t[k], S.x1[k], S.x2[k], X[k], Y[k], S.u[k], s_rare);
+        const RareOut o = rare_pair(S.t[k], S.x1[k], S.x2[k], X[k], Y[k], EP_STAGE_U ? S.u[k] : ~0u, s_rare);
         A.csx += o.dx;
         A.csy += o.dy;
         A.cnt += o.dcnt;
