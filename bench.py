@@ -6,7 +6,9 @@
 
 A step = one whole EP problem of class D (M = 36, 2^37 uniforms; the
 BASELINE.json headline config) split over the N ranks: each rank runs its
-shard kernel (hpl_ep_run_shard) and, for N > 1, the 13-word NCCL allreduce.
+shard kernel; for N > 1 the 13-word partials are combined inside that kernel
+over peer memory (--combine fused, hpl_ep_run_fused, the default) or by one
+NCCL allreduce after it (--combine nccl).
 EP reads no input arrays (only the (M, seed, a) scalars and a 368-B jump table
 passed as kernel parameters), so "resident in HBM" is vacuous; L2 is flushed
 between timed steps anyway.  Device time: CUDA events per step on the
@@ -200,14 +202,34 @@ def run_ours(args, M):
     out = torch.empty(13, dtype=torch.float64, device=dev)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # > 126 MB L2
 
+    # N > 1 combine: "fused" = the kernel's last block exchanges the 13-word
+    # partials over peer memory (hpl_ep_run_fused); "nccl" = kernel
+    # then one all_reduce.  fused falls back to nccl if peer mapping fails.
+    combine, combine_note, fc = ("none" if world == 1 else args.combine), None, None
+    if combine == "fused":
+        try:
+            fc = multi.FusedComm(dev)
+        except Exception as e:  # e.g. no CUDA IPC / peer access between these GPUs
+            combine, combine_note = "nccl", "fused unavailable: %s" % str(e)[:200]
+        if world > 1:  # every rank must agree on the combine
+            flag = torch.tensor([1.0 if combine == "fused" else 0.0], device=dev)
+            dist.all_reduce(flag, op=dist.ReduceOp.MIN)
+            if flag.item() == 0.0 and combine == "fused":
+                combine, combine_note = "nccl", "fused unavailable on a peer rank"
+
     def step():
-        hpl.hpl_ep_run_shard(M, NPB_SEED, NPB_A, rank, world, out.data_ptr(), stream.cuda_stream)
+        if combine == "fused":
+            fc.run(M, NPB_SEED, NPB_A, out)
+        else:
+            hpl.hpl_ep_run_shard(M, NPB_SEED, NPB_A, rank, world, out.data_ptr(), stream.cuda_stream)
 
     for _ in range(args.warmup):
         step()
-        if world > 1:
+        if combine == "nccl":
             dist.all_reduce(out)
     torch.cuda.synchronize(dev)
+    if combine == "fused":
+        fc.status()  # raises if a warm-up combine timed out
 
     # ---- device-timed region
     sampler = ClockSampler(gpu)
@@ -223,7 +245,7 @@ def run_ours(args, M):
         e0.record(stream)
         step()
         e1.record(stream)
-        if world > 1:
+        if combine == "nccl":
             dist.all_reduce(out)
         e2.record(stream)
         e2.synchronize()
@@ -255,6 +277,8 @@ def run_ours(args, M):
         t0 = time.perf_counter()
         if world == 1:
             sx, sy, q = hpl.hpl_ep_run(M, NPB_SEED, NPB_A)  # blocking, 104-B D2H inside
+        elif combine == "fused":
+            multi.ep_run_fused(fc, M, NPB_SEED, NPB_A)
         else:
             multi.ep_run_distributed(M, NPB_SEED, NPB_A, device=dev)
         e2e_ms.append((time.perf_counter() - t0) * 1e3)
@@ -284,7 +308,11 @@ def run_ours(args, M):
             "data": "synthetic (NPB LCG stream, seed 271828183, a=5^13)",
             "config": {"workload": "NPB EP class %s (M=%d)" % (args.cls, M), "M": M,
                        "global_pairs": 1 << M, "seed": NPB_SEED, "a": NPB_A,
-                       "parallelism": "shard x%d + allreduce(13 x f64)" % world if world > 1 else "1 GPU",
+                       "parallelism": ("1 GPU" if world == 1 else
+                                       "shard x%d + in-kernel combine (peer stores)" % world
+                                       if combine == "fused" else
+                                       "shard x%d + allreduce(13 x f64)" % world),
+                       "combine": combine if combine_note is None else "%s (%s)" % (combine, combine_note),
                        "l2": "flushed (256 MB write) between timed steps; EP reads no inputs",
                        "kernel_shape": list(hpl.hpl_ep_launch_shape(pairs_per_launch))},
             "paper_context": PAPER_CONTEXT,
@@ -306,6 +334,8 @@ def run_ours(args, M):
         if not args.no_cpu_baseline and world == 1:
             line["cpu_baseline"] = cpu_baseline_sample(M, args.cpu_budget)
         print(json.dumps(line), flush=True)
+    if fc is not None:
+        fc.close()
     if world > 1:
         dist.barrier()
         dist.destroy_process_group()
@@ -322,6 +352,8 @@ def main():
     ap.add_argument("--cpu-budget", type=float, default=15.0, help="seconds of oracle work for cpu_baseline")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--ref-batches", type=int, default=0, help="NPB batches per --impl reference step")
+    ap.add_argument("--combine", choices=["fused", "nccl"], default="fused",
+                    help="N>1: in-kernel peer-memory combine (default) or kernel + NCCL all_reduce")
     ap.add_argument("--dist-backend", choices=["nccl", "gloo"], default="nccl",
                     help="gloo only to exercise the N>1 code path with several ranks on one GPU")
     args = ap.parse_args()

@@ -140,6 +140,45 @@ int hpl_ep_run_range(uint64_t seed, uint64_t a, uint64_t pair_begin, uint64_t np
  * uses, copied to host_out[0..n-1].  Blocking.  n <= 2^28. */
 int hpl_lcg_states(uint64_t seed, uint64_t a, uint64_t offset, uint64_t n, uint64_t* host_out);
 
+/* ---- fused cross-GPU combine ----------------------------
+ * EP's only exchange step is the sum of the ranks' 13-word partials
+ * (PAPER.md:1264-1270 names multi-node/multi-GPU as the next step; SURVEY
+ * §8(e)).  Instead of a separate allreduce, hpl_ep_run_fused's kernel does
+ * it itself: its last block stores the shard's partial into slot [rank] of
+ * every rank's inbox (device memory of that rank's GPU, mapped into this
+ * process with CUDA IPC; peer stores over NVLink), signals each inbox with a
+ * system-scope release add, waits (acquire) until its own inbox holds all
+ * nranks partials of this call, and sums them in rank order into dev_out13.
+ * Every rank therefore ends with the same, bitwise reproducible result.
+ * Setup, one process per GPU (or several processes sharing one GPU):
+ *   1. hpl_comm_create(&c, rank, nranks, device, handle) on every rank;
+ *   2. exchange the HPL_COMM_HANDLE_BYTES handles (e.g. an all_gather over
+ *      torch.distributed) into `handles` (nranks * 64 bytes, rank order);
+ *   3. hpl_comm_open(c, handles).
+ * All ranks must then issue the same sequence of hpl_ep_run_fused calls
+ * (same M, seed, a).  Ownership: the comm owns its inbox and mappings;
+ * hpl_comm_free releases them (after the caller's streams are idle). */
+#define HPL_COMM_HANDLE_BYTES 64
+#define HPL_COMM_MAX_RANKS 8
+typedef struct hpl_comm_s* hpl_comm;
+/* nranks in [1, 8], 0 <= rank < nranks; device -1 = current.  Writes the
+ * 64-byte IPC handle of this rank's inbox to handle_out. */
+int hpl_comm_create(hpl_comm* out, int rank, int nranks, int device, void* handle_out);
+/* Map the peers' inboxes (handles in rank order; this rank's own entry is
+ * ignored).  HPL_ESTATE if already open, HPL_ECUDA if a mapping fails. */
+int hpl_comm_open(hpl_comm c, const void* handles);
+/* Wait limit of the in-kernel combine (default 10 s).  A call that times out
+ * writes NaN to word 0 and is counted in hpl_comm_status. */
+int hpl_comm_set_timeout(hpl_comm c, double seconds);
+int hpl_comm_free(hpl_comm c);
+/* EP shard c.rank of c.nranks (pairs [rank 2^M/n, (rank+1) 2^M/n)) with the
+ * in-kernel combine: dev_out13 (13 doubles on c's device) receives the WHOLE
+ * problem's result on every rank.  Asynchronous on `stream`. */
+int hpl_ep_run_fused(hpl_comm c, int M, uint64_t seed, uint64_t a, double* dev_out13, void* stream);
+/* Synchronize `stream`; report the number of fused calls issued (epoch) and
+ * of calls whose combine timed out.  Returns HPL_ECUDA if timeouts > 0. */
+int hpl_comm_status(hpl_comm c, void* stream, uint64_t* epoch, uint64_t* timeouts);
+
 /* ---- reduction -----------------------------------------
  * The paper's fifth benchmark, "the addition of 16M single-precision floating
  * point values" (SHOC): *dev_out =

@@ -77,6 +77,24 @@ struct EPPartial {
   unsigned long long big;  // l >= 10 (HPL_ERANGE)
 };
 
+// ---- fused cross-GPU combine ---------------------------
+// Every rank owns one CommInbox in its own device memory; peers write into it
+// over NVLink (CUDA IPC mappings).  slot[epoch & 1][r] holds rank r's 13-word
+// partial {sx, sy, q0..q9, big}; `arrived` counts partials (system-scope
+// atomic adds, monotonic over calls: after call e it is e * nranks).
+constexpr int COMM_MAX_RANKS = 8;
+struct CommInbox {
+  double slot[2][COMM_MAX_RANKS][16];
+  unsigned long long arrived;
+  unsigned long long timeouts;  // calls whose wait gave up (peer missing)
+};
+struct CommParams {
+  CommInbox* inbox[COMM_MAX_RANKS];  // peer inboxes mapped into this process (own at [rank])
+  int rank, nranks;                   // nranks == 0: no fused combine
+  unsigned long long epoch;           // 1, 2, ... per fused call of this comm
+  unsigned long long timeout_ns;      // give up waiting after this long (word 0 := NaN)
+};
+
 struct EPParams {
   uint64_t jump[NJUMP];  // a^(2^i) mod 2^46
   double coef[6];        // lean constants (kept in the parameter bank, not registers)
@@ -91,6 +109,7 @@ struct EPParams {
   EPPartial* partials;   // [gridDim.x]
   unsigned int* counter; // last-block-done ticket, left at 0 after each launch
   double* out13;         // result
+  CommParams comm;       // fused cross-GPU combine (comm.nranks == 0: off)
 };
 
 }  // namespace hplep

@@ -368,6 +368,9 @@ constexpr int kLoopUnroll = EP_LOOP_UNROLL;  // (#pragma arguments are not macro
 #ifndef EP_ABL
 #define EP_ABL 0       // ablation bit set for timing studies only (results are wrong if != 0)
 #endif
+#ifndef EP_IDX_FUSED
+#define EP_IDX_FUSED 0 // 1: table index clamped before the shift (fused add + min)
+#endif
 #ifndef EP_STAGE_U
 #define EP_STAGE_U 1   // 1: the stage keeps the table index for the rare path (register-allocation knob)
 #endif
@@ -425,8 +428,14 @@ __device__ __forceinline__ void gen_stage(unsigned& vlo, unsigned& vhi, const EP
 #else
     S.t[k] = __dadd_rn(__dmul_rn(S.x1[k], S.x1[k]), __dmul_rn(S.x2[k], S.x2[k]));
 #endif
+#if EP_IDX_FUSED
+    // clamp before the shift (same index; lets ptxas fuse add + min: VIADDMNMX)
+    constexpr unsigned LIM = ((EP_PRED_MODE == 1 ? LOG_TINY : LOG_N) << LOG_SHIFT) | ((1u << LOG_SHIFT) - 1);
+    S.u[k] = min(static_cast<unsigned>(__double2hiint(S.t[k])) + LOG_ADD, LIM) >> LOG_SHIFT;
+#else
     S.u[k] = min((static_cast<unsigned>(__double2hiint(S.t[k])) + LOG_ADD) >> LOG_SHIFT,
                  EP_PRED_MODE == 1 ? LOG_TINY : LOG_N);
+#endif
   }
 #pragma unroll
   for (int k = 0; k < W; ++k) {
@@ -858,10 +867,54 @@ ep_kernel(const __grid_constant__ EPParams P) {
     }
   }
   __syncthreads();
+  if (P.comm.nranks > 0) {
+    // F3: the cross-GPU combine in the same kernel.  Store this shard's 13
+    // words into slot [parity][rank] of every rank's inbox (NVLink peer
+    // stores), fence at system scope, signal each inbox, then wait for all
+    // partials in the own inbox and fold them in rank order (deterministic,
+    // identical on every rank).  No separate collective is launched.
+    const CommParams& C = P.comm;
+    const unsigned par = unsigned(C.epoch & 1), n = unsigned(C.nranks);
+    if (tid < 13 * n) {
+      const unsigned r = tid / 13, w = tid % 13;
+      volatile double* dst = &C.inbox[r]->slot[par][C.rank][w];
+      *dst = s_fin[w];
+    }
+    __threadfence_system();
+    __syncthreads();
+    if (tid < n) {
+      unsigned long long* ctr = &C.inbox[tid]->arrived;
+      asm volatile("red.release.sys.global.add.u64 [%0], 1;" ::"l"(ctr) : "memory");
+    }
+    if (tid == 0) {
+      const unsigned long long want = C.epoch * n;
+      unsigned long long* own = &C.inbox[C.rank]->arrived;
+      unsigned long long t0, now, v;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+      int timed_out = 0;
+      for (;;) {
+        asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(own) : "memory");
+        if (v >= want) break;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(now));
+        if (now - t0 > C.timeout_ns) { timed_out = 1; break; }
+        __nanosleep(200);
+      }
+      if (timed_out) atomicAdd(&C.inbox[C.rank]->timeouts, 1ull);
+      s_last = timed_out;  // reuse: 1 = combine failed
+    }
+    __syncthreads();
+    if (tid < 13) {
+      const volatile double* src = &C.inbox[C.rank]->slot[par][0][tid];
+      double acc = 0.0;
+      for (unsigned r = 0; r < n; ++r) acc += src[r * 16];  // rank order
+      s_fin[tid] = acc;
+    }
+    __syncthreads();
+  }
   if (tid == 0) {
     double gc = 0.0;
     for (int k = 0; k < 10; ++k) gc += s_fin[2 + k];  // exact integer sum
-    const bool big = s_fin[12] != 0.0;
+    const bool big = s_fin[12] != 0.0 || (P.comm.nranks > 0 && s_last != 0);
     P.out13[0] = big ? __longlong_as_double(0x7FF8000000000000ll) : s_fin[0];
     P.out13[1] = s_fin[1];
     for (int k = 0; k < 10; ++k) P.out13[2 + k] = s_fin[2 + k];
@@ -1101,7 +1154,7 @@ int launch_shape(int device, uint64_t npairs, const EPConfig& cfg, int* blocks, 
 }
 
 int launch_ep(int device, uint64_t seed, uint64_t a, uint64_t pair_begin, uint64_t npairs,
-              const EPConfig& cfg, double* dev_out13, cudaStream_t stream) {
+              const EPConfig& cfg, double* dev_out13, cudaStream_t stream, const CommParams* comm) {
   const LogEntry* tab;
   int sms;
   int rc = device_state(device, &tab, &sms);
@@ -1124,6 +1177,7 @@ int launch_ep(int device, uint64_t seed, uint64_t a, uint64_t pair_begin, uint64
   P.partials = partials;
   P.counter = counter;
   P.out13 = dev_out13;
+  if (comm) P.comm = *comm;
 
   const bool a32 = (a >> 32) == 0;
   pick_kernel(cfg.variant, a32, threads)<<<blocks, threads, smem, stream>>>(P);

@@ -34,7 +34,8 @@ uint64_t host_jump(uint64_t x, uint64_t k, const uint64_t* J);
 
 int launch_shape(int device, uint64_t npairs, const EPConfig& cfg, int* blocks, int* threads, int* smem);
 int launch_ep(int device, uint64_t seed, uint64_t a, uint64_t pair_begin, uint64_t npairs,
-              const EPConfig& cfg, double* dev_out13, cudaStream_t stream);
+              const EPConfig& cfg, double* dev_out13, cudaStream_t stream,
+              const CommParams* comm = nullptr);
 int launch_lcg_states(uint64_t seed, uint64_t a, uint64_t offset, uint64_t n, uint64_t* dev_out,
                       cudaStream_t stream);
 unsigned long long launch_count();

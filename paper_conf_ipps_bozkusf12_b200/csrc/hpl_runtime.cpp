@@ -288,6 +288,123 @@ int hpl_ep_run_shard(int M, uint64_t seed, uint64_t a, int rank, int nranks, dou
   return hpl_ep_run_range(seed, a, begin, n, dev_out13, stream);
 }
 
+// ---- fused cross-GPU combine ------------------------------
+struct hpl_comm_s {
+  int rank = 0, nranks = 0, device = -1;
+  hplep::CommInbox* own = nullptr;                  // cudaMalloc'd on `device`
+  hplep::CommInbox* peer[hplep::COMM_MAX_RANKS] = {};  // mapped (own at [rank])
+  bool opened = false;
+  unsigned long long epoch = 0;
+  unsigned long long timeout_ns = 10ull * 1000000000ull;
+};
+
+int hpl_comm_create(hpl_comm* out, int rank, int nranks, int device, void* handle_out) {
+  if (!out || !handle_out) return set_error(HPL_EINVAL, "NULL argument");
+  if (nranks < 1 || nranks > hplep::COMM_MAX_RANKS) return set_error(HPL_EINVAL, "nranks must be in [1, %d]", hplep::COMM_MAX_RANKS);
+  if (rank < 0 || rank >= nranks) return set_error(HPL_EINVAL, "rank out of range");
+  if (device < 0) {
+    int rc = current_device(&device);
+    if (rc) return rc;
+  }
+  DeviceGuard g(device);
+  if (g.rc) return g.rc;
+  hpl_comm c = new (std::nothrow) hpl_comm_s;
+  if (!c) return set_error(HPL_ENOMEM, "comm");
+  c->rank = rank;
+  c->nranks = nranks;
+  c->device = device;
+  cudaError_t e = cudaMalloc(&c->own, sizeof(hplep::CommInbox));
+  if (e == cudaSuccess) e = cudaMemset(c->own, 0, sizeof(hplep::CommInbox));
+  if (e == cudaSuccess) e = cudaDeviceSynchronize();
+  cudaIpcMemHandle_t h;
+  if (e == cudaSuccess) e = cudaIpcGetMemHandle(&h, c->own);
+  if (e != cudaSuccess) {
+    if (c->own) cudaFree(c->own);
+    delete c;
+    return set_cuda_error(e, "comm inbox");
+  }
+  static_assert(sizeof(cudaIpcMemHandle_t) == HPL_COMM_HANDLE_BYTES, "IPC handle size");
+  std::memcpy(handle_out, &h, sizeof(h));
+  c->peer[rank] = c->own;
+  *out = c;
+  return HPL_OK;
+}
+
+int hpl_comm_open(hpl_comm c, const void* handles) {
+  if (!c || !handles) return set_error(HPL_EINVAL, "NULL argument");
+  if (c->opened) return set_error(HPL_ESTATE, "comm already open");
+  DeviceGuard g(c->device);
+  if (g.rc) return g.rc;
+  const unsigned char* hb = static_cast<const unsigned char*>(handles);
+  for (int r = 0; r < c->nranks; ++r) {
+    if (r == c->rank) continue;
+    cudaIpcMemHandle_t h;
+    std::memcpy(&h, hb + size_t(r) * HPL_COMM_HANDLE_BYTES, sizeof(h));
+    void* p = nullptr;
+    cudaError_t e = cudaIpcOpenMemHandle(&p, h, cudaIpcMemLazyEnablePeerAccess);
+    if (e != cudaSuccess) {
+      for (int q = 0; q < r; ++q)
+        if (q != c->rank && c->peer[q]) { cudaIpcCloseMemHandle(c->peer[q]); c->peer[q] = nullptr; }
+      return set_cuda_error(e, "cudaIpcOpenMemHandle (peer inbox)");
+    }
+    c->peer[r] = static_cast<hplep::CommInbox*>(p);
+  }
+  c->opened = true;
+  return HPL_OK;
+}
+
+int hpl_comm_set_timeout(hpl_comm c, double seconds) {
+  if (!c || !(seconds > 0.0) || seconds > 3600.0) return set_error(HPL_EINVAL, "timeout must be in (0, 3600] s");
+  c->timeout_ns = static_cast<unsigned long long>(seconds * 1e9);
+  return HPL_OK;
+}
+
+int hpl_comm_free(hpl_comm c) {
+  if (!c) return HPL_OK;
+  DeviceGuard g(c->device);
+  for (int r = 0; r < c->nranks; ++r)
+    if (r != c->rank && c->peer[r]) cudaIpcCloseMemHandle(c->peer[r]);
+  if (c->own) cudaFree(c->own);
+  delete c;
+  return HPL_OK;
+}
+
+int hpl_ep_run_fused(hpl_comm c, int M, uint64_t seed, uint64_t a, double* dev_out13, void* stream) {
+  if (!c || !dev_out13) return set_error(HPL_EINVAL, "NULL argument");
+  if (!c->opened) return set_error(HPL_ESTATE, "comm not opened (hpl_comm_open)");
+  uint64_t begin, n;
+  int rc = shard_range(M, c->rank, c->nranks, &begin, &n);
+  if (!rc) rc = validate(seed, a);
+  if (rc) return rc;
+  DeviceGuard g(c->device);
+  if (g.rc) return g.rc;
+  hplep::CommParams cp;
+  std::memset(&cp, 0, sizeof(cp));
+  for (int r = 0; r < c->nranks; ++r) cp.inbox[r] = c->peer[r];
+  cp.rank = c->rank;
+  cp.nranks = c->nranks;
+  cp.epoch = c->epoch + 1;
+  cp.timeout_ns = c->timeout_ns;
+  rc = launch_ep(c->device, seed, a, begin, n, t_cfg, dev_out13, static_cast<cudaStream_t>(stream), &cp);
+  if (rc) return rc;
+  c->epoch += 1;  // only launched calls advance the epoch
+  return HPL_OK;
+}
+
+int hpl_comm_status(hpl_comm c, void* stream, uint64_t* epoch, uint64_t* timeouts) {
+  if (!c || !epoch || !timeouts) return set_error(HPL_EINVAL, "NULL argument");
+  DeviceGuard g(c->device);
+  if (g.rc) return g.rc;
+  cudaError_t e = cudaStreamSynchronize(static_cast<cudaStream_t>(stream));
+  unsigned long long t = 0;
+  if (e == cudaSuccess) e = cudaMemcpy(&t, &c->own->timeouts, sizeof(t), cudaMemcpyDeviceToHost);
+  if (e != cudaSuccess) return set_cuda_error(e, "comm status");
+  *epoch = c->epoch;
+  *timeouts = t;
+  if (t) return set_error(HPL_ECUDA, "fused combine: %llu call(s) timed out waiting for a peer", t);
+  return HPL_OK;
+}
+
 int hpl_ep_eval(int M, uint64_t seed, uint64_t a, int rank, int nranks, hpl_array out13) {
   if (!out13) return set_error(HPL_EINVAL, "out13 is NULL");
   if (out13->t != HPL_F64 || out13->count != 13) return set_error(HPL_EINVAL, "out13 must be an HPL_F64 array of 13 elements");

@@ -34,7 +34,10 @@ EXPORTS = (
     "hpl_lcg_states", "hpl_ep_set_config", "hpl_ep_launch_shape", "hpl_ep_launch_count",
     "hpl_eval", "hpl_kernel_count", "hpl_kernel_info", "hpl_reduce_sum_f32",
     "hpl_ep_pairs_debug",
+    "hpl_comm_create", "hpl_comm_open", "hpl_comm_set_timeout", "hpl_comm_free",
+    "hpl_ep_run_fused", "hpl_comm_status",
 )
+HPL_COMM_HANDLE_BYTES, HPL_COMM_MAX_RANKS = 64, 8
 HPL_ARG_ARRAY, HPL_ARG_F64, HPL_ARG_F32, HPL_ARG_I64, HPL_ARG_I32 = 0, 1, 2, 3, 4
 
 
@@ -92,6 +95,12 @@ def _load() -> ctypes.CDLL:
         "hpl_reduce_sum_f32": (c_int, [c_void_p, c_i64, c_void_p, c_void_p]),
         "hpl_ep_pairs_debug": (c_int, [c_u64, c_u64, c_u64, c_u64, P(c_double)]),
         "hpl_kernel_info": (c_int, [c_int, P(ctypes.c_char_p), P(ctypes.c_char_p)]),
+        "hpl_comm_create": (c_int, [P(c_void_p), c_int, c_int, c_int, c_void_p]),
+        "hpl_comm_open": (c_int, [c_void_p, c_void_p]),
+        "hpl_comm_set_timeout": (c_int, [c_void_p, c_double]),
+        "hpl_comm_free": (c_int, [c_void_p]),
+        "hpl_ep_run_fused": (c_int, [c_void_p, c_int, c_u64, c_u64, c_void_p, c_void_p]),
+        "hpl_comm_status": (c_int, [c_void_p, c_void_p, P(c_u64), P(c_u64)]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)
@@ -226,6 +235,42 @@ def hpl_ep_launch_count() -> int:
     c = ctypes.c_uint64()
     _check(_load().hpl_ep_launch_count(ctypes.byref(c)), "hpl_ep_launch_count")
     return c.value
+
+
+# ------------------------------------------------ fused combine (F3)
+def hpl_comm_create(rank: int, nranks: int, device: int = -1) -> tuple[int, bytes]:
+    """Create this rank's inbox; returns (comm handle, 64-byte IPC handle)."""
+    c = ctypes.c_void_p()
+    buf = ctypes.create_string_buffer(HPL_COMM_HANDLE_BYTES)
+    _check(_load().hpl_comm_create(ctypes.byref(c), rank, nranks, device, buf), "hpl_comm_create")
+    return c.value, buf.raw
+
+
+def hpl_comm_open(comm: int, handles: bytes) -> None:
+    """handles: nranks * 64 bytes in rank order."""
+    buf = ctypes.create_string_buffer(bytes(handles), len(handles))
+    _check(_load().hpl_comm_open(comm, buf), "hpl_comm_open")
+
+
+def hpl_comm_set_timeout(comm: int, seconds: float) -> None:
+    _check(_load().hpl_comm_set_timeout(comm, seconds), "hpl_comm_set_timeout")
+
+
+def hpl_comm_free(comm: int) -> None:
+    _check(_load().hpl_comm_free(comm), "hpl_comm_free")
+
+
+def hpl_ep_run_fused(comm: int, M: int, seed: int, a: int, dev_out13: int,
+                     stream: int | None = None) -> None:
+    _check(_load().hpl_ep_run_fused(comm, M, seed, a, dev_out13, stream or None), "hpl_ep_run_fused")
+
+
+def hpl_comm_status(comm: int, stream: int | None = None) -> tuple[int, int]:
+    """(epoch, timeouts) after synchronizing `stream`; raises if a combine timed out."""
+    e, t = ctypes.c_uint64(), ctypes.c_uint64()
+    _check(_load().hpl_comm_status(comm, stream or None, ctypes.byref(e), ctypes.byref(t)),
+           "hpl_comm_status")
+    return e.value, t.value
 
 
 # ---------------------------------------------------------- reduction (F2)

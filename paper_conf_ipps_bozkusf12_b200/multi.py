@@ -1,4 +1,4 @@
-"""One process per GPU: shard EP by LCG skip-ahead, combine with one allreduce.
+"""One process per GPU: shard EP by LCG skip-ahead, combine the partials.
 
 SURVEY.md §8(e): rank r of G evaluates pairs [r*2^M/G, (r+1)*2^M/G) with
 ``hpl_ep_run_shard`` (its kernel jumps the stream to seed*a^(2 r 2^M/G)); the
@@ -7,6 +7,11 @@ SURVEY.md §8(e): rank r of G evaluates pairs [r*2^M/G, (r+1)*2^M/G) with
 counts stay exact below 2^53).  The paper runs on one device and names
 distributed memory as future work; this is that step for
 one NVSwitch box.
+
+Two combines: ``ep_shard_and_reduce`` (kernel, then one NCCL allreduce) and
+``FusedComm`` (the EP kernel's last block exchanges the
+partials itself over peer memory, ``hpl_ep_run_fused``; torch.distributed only
+carries the one-time exchange of the 64-byte IPC handles).
 
 This module is marshalling and plumbing only: the compute is the CUDA kernel
 behind ``hpl_ep_run_shard``; ``runner`` exists so the gloo CPU tests can drive
@@ -65,4 +70,61 @@ def ep_run_distributed(M: int, seed: int, a: int, device: Optional[torch.device]
     words = out.cpu().tolist()  # 104-byte D2H
     if words[0] != words[0]:
         raise hpl.HPLError(hpl.HPL_ERANGE, "ep_run_distributed", "annulus index >= 10")
+    return hpl.unpack13(words)
+
+
+class FusedComm:
+    """Peer-memory endpoint for ``hpl_ep_run_fused`` (one per rank and device).
+
+    Construction is collective over ``group``: every rank creates its inbox,
+    the 64-byte CUDA IPC handles are all-gathered, and each rank maps its
+    peers' inboxes.  Then every rank must call :meth:`run` with the same
+    arguments; each call's kernel computes the rank's shard and the combined
+    13-word result of the whole problem (identical on all ranks).
+    """
+
+    def __init__(self, device: torch.device, group: Optional[dist.ProcessGroup] = None,
+                 timeout_s: float = 10.0):
+        self.group = group
+        self.world = dist.get_world_size(group) if dist.is_initialized() else 1
+        self.rank = dist.get_rank(group) if dist.is_initialized() else 0
+        self.device = device
+        self.comm, handle = hpl.hpl_comm_create(self.rank, self.world, device.index)
+        if self.world > 1:
+            backend = dist.get_backend(group)
+            on = device if backend == "nccl" else torch.device("cpu")
+            mine = torch.tensor(list(handle), dtype=torch.uint8, device=on)
+            parts = [torch.empty_like(mine) for _ in range(self.world)]
+            dist.all_gather(parts, mine, group=group)
+            handles = b"".join(bytes(p.cpu().tolist()) for p in parts)
+        else:
+            handles = handle
+        hpl.hpl_comm_open(self.comm, handles)
+        hpl.hpl_comm_set_timeout(self.comm, timeout_s)
+
+    def run(self, M: int, seed: int, a: int, out13: torch.Tensor) -> torch.Tensor:
+        """Asynchronous on the current stream of out13's device."""
+        assert out13.is_cuda and out13.dtype == torch.float64 and out13.numel() == 13
+        hpl.hpl_ep_run_fused(self.comm, M, seed, a, out13.data_ptr(),
+                             torch.cuda.current_stream(out13.device).cuda_stream)
+        return out13
+
+    def status(self) -> tuple[int, int]:
+        return hpl.hpl_comm_status(self.comm, torch.cuda.current_stream(self.device).cuda_stream)
+
+    def close(self) -> None:
+        if self.comm:
+            torch.cuda.synchronize(self.device)
+            hpl.hpl_comm_free(self.comm)
+            self.comm = None
+
+
+def ep_run_fused(comm: FusedComm, M: int, seed: int, a: int) -> dict:
+    """Whole EP problem through the fused combine; host result on every rank."""
+    out = torch.empty(13, dtype=torch.float64, device=comm.device)
+    comm.run(M, seed, a, out)
+    words = out.cpu().tolist()  # 104-byte D2H
+    comm.status()
+    if words[0] != words[0]:
+        raise hpl.HPLError(hpl.HPL_ERANGE, "ep_run_fused", "annulus index >= 10")
     return hpl.unpack13(words)
