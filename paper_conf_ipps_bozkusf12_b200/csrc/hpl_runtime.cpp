@@ -8,6 +8,7 @@
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
+#include <deque>
 #include <mutex>
 #include <new>
 #include <vector>
@@ -667,7 +668,7 @@ struct RedWs {
   int sms;
 };
 std::mutex g_red_mu;
-std::vector<RedWs> g_red;
+std::deque<RedWs> g_red;  // deque: references stay valid across push_back
 
 int reduce_workspace(int device, cudaStream_t stream, hplep::ReduceWorkspace** ws, int* sms) {
   std::lock_guard<std::mutex> lk(g_red_mu);
@@ -680,7 +681,7 @@ int reduce_workspace(int device, cudaStream_t stream, hplep::ReduceWorkspace** w
   RedWs w{device, stream, {}, 0};
   cudaError_t e = cudaDeviceGetAttribute(&w.sms, cudaDevAttrMultiProcessorCount, device);
   if (e != cudaSuccess) return set_cuda_error(e, "cudaDeviceGetAttribute");
-  w.ws.capacity = w.sms * 4;
+  w.ws.capacity = w.sms * 16;  // >= blocks of any launch configuration
   e = cudaMalloc(&w.ws.partials, sizeof(double) * w.ws.capacity);
   if (e == cudaSuccess) e = cudaMalloc(&w.ws.counter, sizeof(unsigned));
   if (e == cudaSuccess) e = cudaMemset(w.ws.counter, 0, sizeof(unsigned));

@@ -2,8 +2,9 @@
 // 16M single-precision floating point values" (SHOC,
 // PAPER.md:793-795), as an HBM-bound sm_100a kernel.
 //
-// One launch: a grid sized to the SMs streams the input with 16-byte loads
-// (4 independent float4 per thread per iteration in flight), accumulates in
+// One launch: a grid of at most one resident wave streams the input with
+// 16-byte loads (8 independent float4 per thread per round in flight, the
+// thread count chosen so the rounds cover the input), accumulates in
 // FP64 (reading R11: the sum is defined exactly; FP64 accumulation keeps the
 // error ~1e-14 of sum|x| at any size), then warp shuffle -> per-warp shared
 // memory -> per-block partial -> last-block fixed-order finalize (the EP
@@ -16,7 +17,16 @@
 
 namespace hplep {
 
-constexpr int RED_THREADS = 512;
+#ifndef RED_THREADS_CFG
+#define RED_THREADS_CFG 512
+#endif
+#ifndef RED_UNROLL
+#define RED_UNROLL 8   // independent 16-B loads in flight per thread (4: -25 % at 16M floats)
+#endif
+#ifndef RED_BPS
+#define RED_BPS 2      // blocks per SM (one wave)
+#endif
+constexpr int RED_THREADS = RED_THREADS_CFG;
 
 __global__ void __launch_bounds__(RED_THREADS)
 reduce_sum_f32_kernel(const float* __restrict__ in, int64_t n, double* __restrict__ partials,
@@ -32,13 +42,15 @@ reduce_sum_f32_kernel(const float* __restrict__ in, int64_t n, double* __restric
   if (tid < head) acc += double(__ldcs(in + tid));
   const float4* v = reinterpret_cast<const float4*>(in + head);
   const int64_t nv = (n - head) / 4;
+  // full rounds of RED_UNROLL independent 16-B loads per thread (the grid is
+  // sized so that the rounds cover the input), then a short remainder
   int64_t i = tid;
-  for (; i + 3 * T < nv; i += 4 * T) {  // four independent 16-B loads in flight
-    const float4 a = __ldcs(v + i), b = __ldcs(v + i + T), c = __ldcs(v + i + 2 * T), d = __ldcs(v + i + 3 * T);
-    acc += (double(a.x) + double(a.y)) + (double(a.z) + double(a.w));
-    acc += (double(b.x) + double(b.y)) + (double(b.z) + double(b.w));
-    acc += (double(c.x) + double(c.y)) + (double(c.z) + double(c.w));
-    acc += (double(d.x) + double(d.y)) + (double(d.z) + double(d.w));
+  for (; i + (RED_UNROLL - 1) * T < nv; i += RED_UNROLL * T) {
+    float4 r[RED_UNROLL];
+#pragma unroll
+    for (int k = 0; k < RED_UNROLL; ++k) r[k] = __ldcs(v + i + k * T);
+#pragma unroll
+    for (int k = 0; k < RED_UNROLL; ++k) acc += (double(r[k].x) + double(r[k].y)) + (double(r[k].z) + double(r[k].w));
   }
   for (; i < nv; i += T) {
     const float4 a = __ldcs(v + i);
@@ -80,9 +92,14 @@ reduce_sum_f32_kernel(const float* __restrict__ in, int64_t n, double* __restric
 
 int launch_reduce_sum_f32(const float* in, int64_t n, double* out, ReduceWorkspace& ws, int sms,
                           cudaStream_t stream) {
-  int blocks = sms * 4;  // 2048 threads/SM resident: enough bytes in flight for HBM
-  const int64_t want = (n / 4 + RED_THREADS - 1) / RED_THREADS;
-  if (want < blocks) blocks = want > 0 ? int(want) : 1;
+  // at most one resident wave (sms * RED_BPS blocks); within it, as few
+  // threads as make every thread's work whole rounds of RED_UNROLL loads
+  const int64_t tmax = int64_t(sms) * RED_BPS * RED_THREADS, nv = n / 4;
+  const int64_t rounds = (nv + RED_UNROLL * tmax - 1) / (RED_UNROLL * tmax);
+  const int64_t t = rounds > 0 ? (nv + RED_UNROLL * rounds - 1) / (RED_UNROLL * rounds) : 1;
+  int blocks = int((t + RED_THREADS - 1) / RED_THREADS);
+  if (blocks < 1) blocks = 1;
+  if (blocks > sms * RED_BPS) blocks = sms * RED_BPS;
   if (blocks > ws.capacity) return set_error(HPL_EINVAL, "reduce workspace too small");
   reduce_sum_f32_kernel<<<blocks, RED_THREADS, 0, stream>>>(in, n, ws.partials, ws.counter, out);
   cudaError_t e = cudaGetLastError();

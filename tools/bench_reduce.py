@@ -1,8 +1,10 @@
 """F2 measurement: hpl_reduce_sum_f32 GB/s vs the measured HBM copy peak.
 
 python tools/bench_reduce.py [--n N ...]   (one JSON line per size)
-Inputs are resident in HBM; L2 (126 MB) is flushed by a 256 MB write between
-timed launches; CUDA events on the launching stream.  Algorithmic bytes =
+Inputs are resident in HBM; L2 (126 MB) is flushed between timed launches by
+a 256 MB write followed by a 256 MB read of another buffer (so the write's
+dirty lines are written back before the timed region, not inside it;
+--flush write keeps only the write); CUDA events on the launching stream.  Algorithmic bytes =
 4 n (each float read once; the 8-byte result and ~5 KB of partials ignored).
 """
 import argparse, json, os, sys
@@ -13,6 +15,7 @@ from paper_conf_ipps_bozkusf12_b200 import hpl
 ap = argparse.ArgumentParser()
 ap.add_argument("--n", type=int, nargs="*", default=[16 << 20, 256 << 20])
 ap.add_argument("--iters", type=int, default=10)
+ap.add_argument("--flush", choices=["write", "write_read"], default="write_read")
 a = ap.parse_args()
 root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 pk = json.load(open(os.path.join(root, "MEASURED_PEAKS.json"))) if os.path.exists(os.path.join(root, "MEASURED_PEAKS.json")) else {}
@@ -20,6 +23,7 @@ peak = float(pk.get("hbm_gbs", 6650.0))
 torch.cuda.set_device(0); hpl.hpl_set_device(0)
 s = torch.cuda.current_stream()
 flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+flush_rd = torch.ones(64 << 20, dtype=torch.float32, device="cuda")  # 256 MB, read to clean L2
 for n in a.n:
     x = torch.randn(n, dtype=torch.float32, device="cuda")
     out = torch.empty(1, dtype=torch.float64, device="cuda")
@@ -34,6 +38,8 @@ for n in a.n:
     ts = []
     for _ in range(a.iters):
         flush.zero_()
+        if a.flush == "write_read":
+            flush_rd.sum()
         e0 = torch.cuda.Event(enable_timing=True); e1 = torch.cuda.Event(enable_timing=True)
         e0.record(s)
         g.replay()
@@ -41,7 +47,7 @@ for n in a.n:
         ts.append(e0.elapsed_time(e1) / 1e3)
     t = sorted(ts)[len(ts) // 2]
     gbs = 4 * n / t / 1e9
-    print(json.dumps({"workload": "sum of %d f32 (F2)" % n, "median_s": t, "GB/s": round(gbs, 1),
+    print(json.dumps({"workload": "sum of %d f32 (F2)" % n, "flush": a.flush, "median_s": t, "GB/s": round(gbs, 1),
                       "roofline": {"bound": "hbm", "achieved": round(gbs, 1), "peak": peak, "unit": "GB/s",
                                    "frac": round(gbs / peak, 4), "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy)"},
                       "result": out.item(), "torch_sum_f64": float(x.double().sum())}), flush=True)
