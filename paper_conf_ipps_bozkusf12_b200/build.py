@@ -37,14 +37,15 @@ def _stale() -> bool:
 
 
 def build(force: bool = False, verbose: bool = False, out: str | None = None,
-          defines: tuple = ()) -> str:
-    """Compile libhpl.so.  `out`/`defines` build development A/B variants
-    (e.g. defines=("EP_ILP=4",)) to another path; the product is LIB."""
+          defines: tuple = (), extra: tuple = ()) -> str:
+    """Compile libhpl.so.  `out`/`defines`/`extra` (additional nvcc flags) build
+    development A/B variants (e.g. defines=("EP_ILP=4",)) to another path; the
+    product is LIB."""
     lib = out or LIB
-    if out is None and not defines and not force and not _stale():
+    if out is None and not defines and not extra and not force and not _stale():
         return LIB
     tmp = lib + ".tmp%d" % os.getpid()
-    cmd = [NVCC, *NVCC_FLAGS, *["-D" + d for d in defines], "-I", os.path.join(ROOT, "include"),
+    cmd = [NVCC, *NVCC_FLAGS, *extra, *["-D" + d for d in defines], "-I", os.path.join(ROOT, "include"),
            "-o", tmp, *SOURCES]
     res = subprocess.run(cmd, capture_output=True, text=True)
     log = os.path.join(PKG, "build.log" if out is None else os.path.basename(lib) + ".log")

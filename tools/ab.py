@@ -13,8 +13,10 @@ if sys.argv[1] == "build":
     os.makedirs(OUT, exist_ok=True)
     for spec in sys.argv[2:]:
         name, _, defs = spec.partition("=")
-        d = tuple(x for x in defs.split(";") if x)
-        build.build(out=os.path.join(OUT, "libhpl_%s.so" % name), defines=d)
+        items = [x for x in defs.split(";") if x]
+        d = tuple(x for x in items if not x.startswith("-"))     # -D defines
+        x = tuple(y for x in items if x.startswith("-") for y in x.split())  # extra nvcc flags
+        build.build(out=os.path.join(OUT, "libhpl_%s.so" % name), defines=d, extra=x)
         print("built", name, d)
 else:
     M, threads = sys.argv[2], sys.argv[3]
