@@ -45,6 +45,21 @@ __device__ __forceinline__ double rsqrt_approx(double p) {
   return y;
 }
 
+#ifndef EP_Y0LO
+#define EP_Y0LO 0  // 1: rsqrt seed = {low word of p, MUFU.RSQ64H high word} (no zeroing move)
+#endif
+// MUFU.RSQ64H yields only the high word; rsqrt.approx.f64 zeroes the low word
+// with an extra (IMAD-pipe) move.  Any low word perturbs the seed by < 2^-20
+// relative, below the MUFU's own 2^-20 error, and the cubic Newton step takes
+// a 2^-19 seed to < 2^-56, so the low word of p itself serves.
+__device__ __forceinline__ double rsqrt_seed_hi(double p) {
+  double y;
+  asm("{\n\t.reg .f64 r;\n\t.reg .b32 rl, rh, pl, ph;\n\t"
+      "rsqrt.approx.ftz.f64 r, %1;\n\tmov.b64 {rl, rh}, r;\n\tmov.b64 {pl, ph}, %1;\n\t"
+      "mov.b64 %0, {pl, rh};\n\t}" : "=d"(y) : "d"(p));
+  return y;
+}
+
 // 1 << (8 l) for l in 0..3 in one PRMT (backward-4-extract of the byte string
 // {1,0,0,0,0,0,0,0} starting at byte l); lanes with l >= 4 never use it.
 __device__ __forceinline__ unsigned bin_increment(unsigned l, unsigned one = 1u) {
@@ -490,12 +505,21 @@ __device__ __forceinline__ void transform_stage(const Stage<W>& S, const EPParam
     p[k] = fma(L[k], S.t[k], 0x1p-200);
 #if EP_ABL & 4  // ablation: no MUFU
     y0[k] = S.t[k];
+#elif EP_Y0LO
+    y0[k] = rsqrt_seed_hi(p[k]);
 #else
     y0[k] = rsqrt_approx(p[k]);
 #endif
   }
+#if EP_Y0LO
+  // e = 1 - p y0^2 as 1 - (L y0)(t y0): p is dead after the MUFU (its
+  // register pair can hold y0), g = L y0 is reused below
+#pragma unroll
+  for (int k = 0; k < W; ++k) e[k] = fma(-__dmul_rn(L[k], y0[k]), __dmul_rn(S.t[k], y0[k]), 1.0);
+#else
 #pragma unroll
   for (int k = 0; k < W; ++k) e[k] = fma(-__dmul_rn(p[k], y0[k]), y0[k], 1.0);
+#endif
   bool any_rare = false;
   unsigned sel_min = 0xFFFFFFFFu;
   (void)sel_min;

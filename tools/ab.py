@@ -27,6 +27,6 @@ else:
                             "--threads", threads, "--reps", "3"], env=env, capture_output=True, text=True)
         for line in r.stdout.splitlines():
             d = json.loads(line)
-            print(json.dumps({"variant": n, **{k: d[k] for k in ("thr", "M", "s", "Mops", "gc")}}), flush=True)
+            print(json.dumps({"variant": n, **{k: d[k] for k in ("thr", "M", "s", "Mops", "gc", "sx", "sy") if k in d}}), flush=True)
         if r.returncode:
             print(n, "FAILED", r.stderr[-500:])

@@ -36,4 +36,4 @@ for variant in map(int, a.variants.split(",")):
                 t = min(ts)
                 print(json.dumps({"variant": variant, "thr": thr, "bps": bps, "M": M, "shape": shape,
                                   "s": round(t, 6), "Mops": round((2 << M) / t / 1e6, 1),
-                                  "gc": int(out[12].item())}), flush=True)
+                                  "gc": int(out[12].item()), "sx": out[0].item(), "sy": out[1].item()}), flush=True)
