@@ -60,3 +60,19 @@ def make_csr(n_rows, n_cols, density, seed):
         cols[rowptr[i]:rowptr[i + 1]] = np.sort(rng.choice(n_cols, counts[i], replace=False))
     A = rng.uniform(-1.0, 1.0, int(rowptr[-1])).astype(np.float32)
     return rowptr.astype(np.int32), cols, A
+
+
+# ----------------------------------------------------------- F4: transpose
+# Fig. 7's transpose size: "the transposition of a 16K x 16K matrix"
+# (PAPER.md:949-950), single precision like the AMD SDK kernel it was taken
+# from; Fig. 9's smaller device used 5K x 5K
+# (PAPER.md:1087-1088).
+TRANSPOSE_N = 16 * 1024
+TRANSPOSE_SMALL_N = 5 * 1024
+
+
+def make_matrix(h, w, seed):
+    """Seeded synthetic float32 h x w matrix (row-major), values U(-1, 1);
+    distinct values almost surely, so a misplaced element is detected."""
+    import numpy as np
+    return np.random.default_rng(seed).uniform(-1.0, 1.0, (h, w)).astype(np.float32)

@@ -188,6 +188,20 @@ int hpl_comm_status(hpl_comm c, void* stream, uint64_t* epoch, uint64_t* timeout
  * hpl_eval as "sum_f32" (in:F32:r, out:F64:w). */
 int hpl_reduce_sum_f32(const float* dev_in, int64_t n, double* dev_out, void* stream);
 
+/* ---- matrix transpose -----------------------------------
+ * The paper's transpose benchmark, "the transposition of a 16K x 16K matrix"
+ * (AMD APP SDK; blocked through local
+ * memory; Fig. 10(b) dest[idy][idx] = src[idx][idy],
+ * PAPER.md:1132-1138): dev_dst[j*h + i] = dev_src[i*w + j] for i < h, j < w,
+ * i.e. src is h x w and dst is w x h, both row-major float32 in device memory
+ * of the current device; asynchronous on `stream`.  Both pointers 4-byte
+ * aligned (16-byte aligned src with w % 4 == 0 takes the vector path); the
+ * ranges must not overlap (EINVAL: no in-place transpose); h * w == 0 is a
+ * no-op.  Bit-exact (data movement only).  Also registered for hpl_eval as
+ * "transpose_f32" (dest:F32:w, src:F32:r) over dest's 2-D domain
+ * (global = {w, h}); the local domain is not used (64 x 64 tiles). */
+int hpl_transpose_f32(const float* dev_src, int64_t h, int64_t w, float* dev_dst, void* stream);
+
 /* ---- generic eval over an index domain ----------------
  * The paper's eval(f).global(..).local(..)(args) for
  * hand-written CUDA kernels registered in the library (HPL captures C++

@@ -15,7 +15,8 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libhpl.so")
-SOURCES = [os.path.join(CSRC, f) for f in ("ep_kernel.cu", "eval_kernels.cu", "reduce_kernel.cu", "hpl_runtime.cpp")]
+SOURCES = [os.path.join(CSRC, f) for f in ("ep_kernel.cu", "eval_kernels.cu", "reduce_kernel.cu", "transpose_kernel.cu",
+                                                 "hpl_runtime.cpp")]
 HEADERS = [os.path.join(CSRC, f) for f in ("ep_common.cuh", "ep_launch.h", "eval_launch.h", "reduce_launch.h")] + [
     os.path.join(ROOT, "include", "hpl.h")]
 

@@ -708,6 +708,26 @@ int hpl_reduce_sum_f32(const float* dev_in, int64_t n, double* dev_out, void* st
 }
 
 
+int hpl_transpose_f32(const float* dev_src, int64_t h, int64_t w, float* dev_dst, void* stream) {
+  if (h < 0 || w < 0) return set_error(HPL_EINVAL, "h and w must be >= 0");
+  if (h > 0 && w > 0 && h > INT64_MAX / 4 / w) return set_error(HPL_EINVAL, "h * w too large");
+  const int64_t n = h * w;
+  if (n == 0) return HPL_OK;
+  if (!dev_src || !dev_dst) return set_error(HPL_EINVAL, "NULL pointer");
+  if ((reinterpret_cast<uintptr_t>(dev_src) | reinterpret_cast<uintptr_t>(dev_dst)) & 3)
+    return set_error(HPL_EINVAL, "dev_src and dev_dst must be 4-byte aligned");
+  const uintptr_t s0 = reinterpret_cast<uintptr_t>(dev_src), d0 = reinterpret_cast<uintptr_t>(dev_dst);
+  const uintptr_t bytes = uintptr_t(n) * sizeof(float);
+  if (s0 < d0 + bytes && d0 < s0 + bytes) return set_error(HPL_EINVAL, "dev_src and dev_dst overlap (no in-place transpose)");
+  int dev;
+  int rc = current_device(&dev);
+  if (rc) return rc;
+  int sms = 0;
+  cudaError_t e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  if (e != cudaSuccess) return set_cuda_error(e, "cudaDeviceGetAttribute");
+  return hplep::launch_transpose_f32(dev_src, dev_dst, h, w, sms, static_cast<cudaStream_t>(stream));
+}
+
 int hpl_ep_pairs_debug(uint64_t seed, uint64_t a, uint64_t pair_begin, uint64_t n, double* host_out) {
   int rc = validate(seed, a);
   if (rc) return rc;

@@ -33,6 +33,7 @@ EXPORTS = (
     "hpl_ep_eval", "hpl_ep_run", "hpl_ep_run_shard", "hpl_ep_run_range",
     "hpl_lcg_states", "hpl_ep_set_config", "hpl_ep_launch_shape", "hpl_ep_launch_count",
     "hpl_eval", "hpl_kernel_count", "hpl_kernel_info", "hpl_reduce_sum_f32",
+    "hpl_transpose_f32",
     "hpl_ep_pairs_debug",
     "hpl_comm_create", "hpl_comm_open", "hpl_comm_set_timeout", "hpl_comm_free",
     "hpl_ep_run_fused", "hpl_comm_status",
@@ -93,6 +94,7 @@ def _load() -> ctypes.CDLL:
         "hpl_eval": (c_int, [ctypes.c_char_p, c_int, P(c_i64), P(c_i64), c_int, P(HplArg)]),
         "hpl_kernel_count": (c_int, [P(c_int)]),
         "hpl_reduce_sum_f32": (c_int, [c_void_p, c_i64, c_void_p, c_void_p]),
+        "hpl_transpose_f32": (c_int, [c_void_p, c_i64, c_i64, c_void_p, c_void_p]),
         "hpl_ep_pairs_debug": (c_int, [c_u64, c_u64, c_u64, c_u64, P(c_double)]),
         "hpl_kernel_info": (c_int, [c_int, P(ctypes.c_char_p), P(ctypes.c_char_p)]),
         "hpl_comm_create": (c_int, [P(c_void_p), c_int, c_int, c_int, c_void_p]),
@@ -276,6 +278,12 @@ def hpl_comm_status(comm: int, stream: int | None = None) -> tuple[int, int]:
 # ---------------------------------------------------------- reduction (F2)
 def hpl_reduce_sum_f32(dev_in: int, n: int, dev_out: int, stream: int | None = None) -> None:
     _check(_load().hpl_reduce_sum_f32(dev_in, n, dev_out, stream or None), "hpl_reduce_sum_f32")
+
+
+# ---------------------------------------------------------- transpose (F4)
+def hpl_transpose_f32(dev_src: int, h: int, w: int, dev_dst: int, stream: int | None = None) -> None:
+    """dev_dst (w x h) = transpose of dev_src (h x w), row-major float32, device pointers."""
+    _check(_load().hpl_transpose_f32(dev_src, h, w, dev_dst, stream or None), "hpl_transpose_f32")
 
 
 # ------------------------------------------------------- generic eval (F1)
