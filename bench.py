@@ -46,6 +46,7 @@ ALG_OPS_ALWAYS = 6
 ALG_OPS_ACCEPTED = 18
 P_ACCEPT = 0.7853981633974483
 ALG_OPS_PER_PAIR = ALG_OPS_ALWAYS + P_ACCEPT * ALG_OPS_ACCEPTED
+EXEC_FP64_PER_PAIR = 22             # SASS of the hot loop (tools/sass_hot.py): DFMA 10 + DMUL 7 + DADD 5
 FP64_LANES_PER_SM_CLK = 64          # measured: tools/probe_fp64.cu (63.9-64.1 lane-DFMA/clk/SM)
 EP_PARAM_BYTES = 560                 # EPParams kernel-parameter block (jump table, a^k table, coefs, scalars)
 
@@ -56,6 +57,15 @@ def peaks():
     if os.path.exists(path):
         p = json.load(open(path))
     return p
+
+
+def load_profile_field(key):
+    """One field of the committed ncu summary of the EP kernel, or None."""
+    path = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    try:
+        return json.load(open(path)).get(key)
+    except Exception:
+        return None
 
 
 def load_profile_traffic():
@@ -322,7 +332,12 @@ def run_ours(args, M):
                          "alg_ops_per_pair": round(ALG_OPS_PER_PAIR, 3),
                          "peak_basis": "%d SMs x %d FP64 lanes/clk x %.0f MHz (sm_max_mhz)"
                                        % (props.multi_processor_count, FP64_LANES_PER_SM_CLK, sm_max),
-                         "kernel_ms": round(kern_avg_s * 1e3, 4)},
+                         "kernel_ms": round(kern_avg_s * 1e3, 4),
+                         # the FP64-issue view: FP64 instructions the kernel
+                         # executes per pair (every pair runs the transform) / peak
+                         "executed_fp64_per_pair": EXEC_FP64_PER_PAIR,
+                         "fp64_pipe_frac": round(achieved / peak_ops * EXEC_FP64_PER_PAIR / ALG_OPS_PER_PAIR, 4),
+                         "ncu_fp64_pipe_active_pct": load_profile_field("fp64_pipe_active_pct")},
             "e2e": {"value": round(units * args.steps / (e2e_tot / 1e3) / 1e6, 1), "unit": UNIT,
                     "h2d_bytes_per_step": EP_PARAM_BYTES * world, "d2h_bytes_per_step": 104 * world,
                     "note": "h2d = kernel-parameter block (jump table + scalars); d2h = 13-word result"},

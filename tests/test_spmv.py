@@ -100,10 +100,31 @@ def test_fig5_toy(gpu, M):
 
 
 @pytest.mark.gpu
-@pytest.mark.parametrize("M", [8, 32])
+@pytest.mark.parametrize("M", [8, 32, 2])
 def test_fig7_size(gpu, M):
     """Fig. 7's spmv: 16K x 16K, 1 % nonzeros."""
     rowptr, cols, A = make_csr(SPMV_ROWS, SPMV_ROWS, SPMV_DENSITY, seed=16)
     vec = np.random.default_rng(17).uniform(-1, 1, SPMV_ROWS).astype(np.float32)
     got = run_spmv(gpu, rowptr, cols, A, vec, M)
     assert np.array_equal(got, osp.hpl_fig5b(rowptr, cols, A, vec, M))
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("M", [4, 32])
+def test_vec_too_large_for_shared_memory(gpu, M):
+    """A wide matrix (80K columns, 320 KB vec, sparse rows: many CTAs whose
+    element ranges are shorter than the 16-byte alignment window)."""
+    rowptr, cols, A = make_csr(700, 80_000, 0.002, seed=M + 40)
+    vec = np.random.default_rng(M).uniform(-1, 1, 80_000).astype(np.float32)
+    got = run_spmv(gpu, rowptr, cols, A, vec, M)
+    assert np.array_equal(got, osp.hpl_fig5b(rowptr, cols, A, vec, M))
+
+
+@pytest.mark.gpu
+def test_rows_exceed_one_resident_wave(gpu):
+    """Many CTAs (150K rows), a ragged last warp (rows * M not a multiple of
+    32), empty rows and rows of 1-2 elements (unaligned chunk ends)."""
+    rowptr, cols, A = make_csr(150_001, 3000, 0.001, seed=77)
+    vec = np.random.default_rng(78).uniform(-1, 1, 3000).astype(np.float32)
+    got = run_spmv(gpu, rowptr, cols, A, vec, 4)
+    assert np.array_equal(got, osp.hpl_fig5b(rowptr, cols, A, vec, 4))

@@ -1,7 +1,8 @@
 """F4 measurement: spmv_csr on Fig. 7's 16K x 16K, 1 % matrix (dev aid).
 
 Device time per hpl_eval with CUDA events (arrays already device-valid, so no
-transfers are issued), L2 flushed between launches.  Algorithmic bytes =
+transfers are issued), L2 flushed between launches (256 MB write, then a
+256 MB read so the dirty lines are written back before the timed region).  Algorithmic bytes =
 A + cols (8 B per nonzero) + rowptr + vec + out (each read/written once).
 """
 import ctypes, json, os, sys
@@ -29,6 +30,7 @@ hs = [arr(hpl.HPL_F32, A, ctypes.c_float), arr(hpl.HPL_F32, vec, ctypes.c_float)
       arr(hpl.HPL_I32, cols, ctypes.c_int32), arr(hpl.HPL_I32, rowptr, ctypes.c_int32),
       hpl.hpl_array_alloc(hpl.HPL_F32, [rows])]
 flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+flush_rd = torch.ones(64 << 20, dtype=torch.float32, device="cuda")  # 256 MB read: writes back the flush's dirty lines
 s = torch.cuda.default_stream()
 for M in (8, 16, 32):
     for _ in range(3):
@@ -43,7 +45,7 @@ for M in (8, 16, 32):
         hpl.hpl_eval("spmv_csr", hs, global_=[rows * M], local=[M])
     ts = []
     for _ in range(20):
-        flush.zero_(); torch.cuda.synchronize()
+        flush.zero_(); flush_rd.sum(); torch.cuda.synchronize()
         e0 = torch.cuda.Event(enable_timing=True); e1 = torch.cuda.Event(enable_timing=True)
         e0.record(s)
         g.replay()
