@@ -132,7 +132,7 @@ def test_fig3_saxpy(gpu):
 
 
 @pytest.mark.gpu
-@pytest.mark.parametrize("N,M", [(256, 32), (4096, 128), (1 << 20, 256)])
+@pytest.mark.parametrize("N,M", [(256, 32), (4096, 128), (1 << 20, 256), (3 * 1024, 1024), (13 * 64, 64), (8, 1)])
 def test_fig4_dotp(gpu, N, M):
     """Fig. 4: per-group partial dot products through Local
     memory, lane 0 sums in order into pSums[gidx]; host sums nGroup partials."""
