@@ -367,13 +367,15 @@ constexpr int kLoopUnroll = EP_LOOP_UNROLL;  // (#pragma arguments are not macro
 #define EP_PIPE_ORDER 0  // 1: single stage, transform then generate (no ping-pong)
 #endif
 #ifndef EP_TMA_TABLE
-#define EP_TMA_TABLE 0 // 1: load the log table with cp.async.bulk (TMA) + mbarrier: ~2 us
-                       // less per launch, but ptxas then allocates the hot loop's registers
-                       // slightly worse (+0.8 operand reads/pair, -1.5 % at class D)
+#define EP_TMA_TABLE 1 // 1: load the log table with cp.async.bulk (TMA) + mbarrier (one
+                       // thread, one 139-KB stream); 0: strided 16-B loads by all threads
+#endif
+#ifndef EP_TAB_BATCH
+#define EP_TAB_BATCH 8   // table-copy loads in flight per thread (1 = the plain strided loop)
 #endif
 #ifndef EP_TMA_WAIT_LATE
-#define EP_TMA_WAIT_LATE 0  // 1: wait for the table after the skip-ahead instead of before
-#endif
+#define EP_TMA_WAIT_LATE 1  // 1: wait for the table after the skip-ahead instead of before
+#endif                      // (TMA + late wait: +2.8 % at class D over the plain copy, session 3)
 #ifndef EP_T2MODE
 #define EP_T2MODE 1    // 1: t2 = g + g (e cc) instead of g + (g e) cc
 #endif
@@ -689,9 +691,21 @@ ep_kernel(const __grid_constant__ EPParams P) {
   __shared__ __align__(8) unsigned long long s_mbar;
   const unsigned mbar = static_cast<unsigned>(__cvta_generic_to_shared(&s_mbar));
   if (VARIANT == HPL_VARIANT_LEAN && !EP_TMA_TABLE) {
+    // EP_TAB_BATCH independent 16-B loads in flight per thread, then the
+    // stores: ~3 L2 round trips for the 139-KB table instead of ~17
     const double2* src = reinterpret_cast<const double2*>(P.table);
     double2* dst = reinterpret_cast<double2*>(smem_raw);
-    for (unsigned i = tid; i < LOG_TAB; i += blockDim.x) dst[i] = __ldg(src + i);
+    const unsigned nt = blockDim.x;
+#pragma unroll 1
+    for (unsigned i0 = tid; i0 < LOG_TAB; i0 += EP_TAB_BATCH * nt) {
+      double2 v[EP_TAB_BATCH];
+#pragma unroll
+      for (int k = 0; k < EP_TAB_BATCH; ++k)
+        if (i0 + k * nt < LOG_TAB) v[k] = __ldg(src + i0 + k * nt);
+#pragma unroll
+      for (int k = 0; k < EP_TAB_BATCH; ++k)
+        if (i0 + k * nt < LOG_TAB) dst[i0 + k * nt] = v[k];
+    }
   }
   if (VARIANT == HPL_VARIANT_LEAN && EP_TMA_TABLE && tid == 0) {
     constexpr unsigned BYTES = LOG_TAB * sizeof(LogEntry), CHUNK = 32768;
