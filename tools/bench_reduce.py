@@ -60,8 +60,21 @@ for n in a.n:
         e1.record(s); e1.synchronize()
         tt.append(e0.elapsed_time(e1) / 1e3)
     t_torch = sorted(tt)[len(tt) // 2]
+    tf = []
+    rf = torch.empty((), dtype=torch.float32, device="cuda")
+    for _ in range(a.iters):
+        flush.zero_()
+        if a.flush == "write_read":
+            flush_rd.sum()
+        e0 = torch.cuda.Event(enable_timing=True); e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(s)
+        torch.sum(x, dim=0, out=rf)
+        e1.record(s); e1.synchronize()
+        tf.append(e0.elapsed_time(e1) / 1e3)
+    t_torch32 = sorted(tf)[len(tf) // 2]
     print(json.dumps({"workload": "sum of %d f32 (F2)" % n, "flush": a.flush, "median_s": t, "GB/s": round(gbs, 1),
                       "torch_sum_f64_GB/s": round(4 * n / t_torch / 1e9, 1),
+                      "torch_sum_f32_GB/s": round(4 * n / t_torch32 / 1e9, 1),
                       "roofline": {"bound": "hbm", "achieved": round(gbs, 1), "peak": peak, "unit": "GB/s",
                                    "frac": round(gbs / peak, 4), "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy)"},
                       "result": out.item(), "torch_sum_f64": float(x.double().sum())}), flush=True)

@@ -59,5 +59,24 @@ for M in (8, 16, 32):
                       "GFLOP/s": round(2 * nnz / t / 1e9, 1),
                       "roofline": {"bound": "hbm", "achieved": round(byts / t / 1e9, 1), "peak": peak, "unit": "GB/s",
                                    "frac": round(byts / t / 1e9 / peak, 4), "bytes": byts}}), flush=True)
+# context: cuSPARSE SpMV of the same matrix through torch (CSR @ dense vector),
+# same flush and event timing (its order of additions differs: not a parity check)
+Acsr = torch.sparse_csr_tensor(torch.from_numpy(rowptr.astype(np.int64)).cuda(), torch.from_numpy(cols.astype(np.int64)).cuda(),
+                               torch.from_numpy(A).cuda(), size=(rows, rows))
+xv = torch.from_numpy(vec).cuda()
+for _ in range(3):
+    yv = Acsr @ xv
+torch.cuda.synchronize()
+tc = []
+for _ in range(20):
+    flush.zero_(); flush_rd.sum(); torch.cuda.synchronize()
+    e0 = torch.cuda.Event(enable_timing=True); e1 = torch.cuda.Event(enable_timing=True)
+    e0.record(s)
+    yv = Acsr @ xv
+    e1.record(s); e1.synchronize()
+    tc.append(e0.elapsed_time(e1) / 1e3)
+t = sorted(tc)[len(tc) // 2]
+print(json.dumps({"workload": "context: torch CSR @ vector (cuSPARSE), same matrix", "median_s": t,
+                  "GFLOP/s": round(2 * nnz / t / 1e9, 1)}), flush=True)
 for h in hs:
     hpl.hpl_array_free(h)
