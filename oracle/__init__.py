@@ -109,6 +109,14 @@ def states(seed: int, a: int, offset: int, n: int) -> list[int]:
     return list(buf[:n])
 
 
+def states_array(seed: int, a: int, offset: int, n: int):
+    """states() as a numpy uint64 array (same C routine; for scanning large ranges)."""
+    import numpy as np
+    out = np.empty(max(n, 1), dtype=np.uint64)
+    _load().ep_oracle_states(float(seed), float(a), offset, n, out.ctypes.data_as(ctypes.POINTER(ctypes.c_uint64)))
+    return out[:n]
+
+
 def an(a: int, mk: int = 16) -> int:
     return int(_load().ep_oracle_an(float(a), mk))
 

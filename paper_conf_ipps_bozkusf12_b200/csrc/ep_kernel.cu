@@ -256,6 +256,9 @@ __device__ __forceinline__ void lean_pair(unsigned& vlo, unsigned& vhi, const EP
 #ifndef EP_ACC_INT
 #define EP_ACC_INT 1   // 1: acceptance t' <= 1/4 by a 64-bit integer compare of the bits
 #endif
+#ifndef EP_ACC_HI
+#define EP_ACC_HI 1    // 1: acceptance from the high word of t' only (rare path settles hi == bits(1/4));
+#endif                 //    -1.5 instructions/pair, +1.4 % at class D (session 3)
 #ifndef EP_LCG_PAR
 #define EP_LCG_PAR 0   // 1: the 2W uniforms of a group from v by independent a^k multiplies
 #endif
@@ -476,6 +479,12 @@ __device__ __forceinline__ void transform_stage(const Stage<W>& S, const EPParam
   for (int k = 0; k < W; ++k) {
     if (EP_PRED_MODE == 1 && !DBG)
       acc[k] = true;  // decided by the selector below (rejects -> NaN or >= 2^21)
+    else if (EP_ACC_HI && !DBG)
+      // high word only: t' < 1/4 is decided exactly; hi == bits(1/4) holds
+      // t' == 1/4 (L = 0 -> X = Y = 0, bin 0: correct on the fast path) and
+      // rejects just above 1/4, whose L < 0 makes X, Y NaN -> selector says
+      // "rare" -> rare_pair rejects them exactly (t > 0.25)
+      acc[k] = static_cast<unsigned>(__double2hiint(S.t[k])) <= 0x3FD00000u;
     else if (EP_ACC_INT)
       acc[k] = static_cast<unsigned long long>(__double_as_longlong(S.t[k])) <= 0x3FD0000000000000ull;
     else

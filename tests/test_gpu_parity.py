@@ -301,3 +301,24 @@ def test_random_streams(env, oracle_mod, case):
     begin = rng.randrange((1 << 43) - n)
     g = gpu_range(env, seed, a, begin, n)
     assert_parity(g, oracle_mod.run_pairs(seed, a, begin, n))
+
+
+def test_acceptance_boundary_pairs(env, oracle_mod):
+    """Pairs whose t lies just above 1 (t' shares the high word of 1/4 and is
+    rejected: the kernel routes them through the rare path, which rejects
+    them exactly) and just below 1 (accepted, top table bucket), located in
+    the class-S stream with the oracle's own LCG; each is checked inside a
+    2^21-pair range in the bench launch shape (q, gc exact, sums within T1)."""
+    import numpy as np
+    st = oracle_mod.states_array(NPB_SEED, NPB_A, 0, 1 << 24)   # x_1 .. x_{2^24}: 2^23 pairs
+    u = st.astype(np.float64) * 2.0 ** -46
+    x1, x2 = 2.0 * u[0::2] - 1.0, 2.0 * u[1::2] - 1.0
+    t = x1 * x1 + x2 * x2                                          # NPB roundings (no contraction in numpy)
+    above = np.where((t > 1.0) & (t < 1.0 + 2.0 ** -20))[0]
+    below = np.where((t <= 1.0) & (t > 1.0 - 2.0 ** -20))[0]
+    assert len(above) >= 4 and len(below) >= 4
+    for i in list(above[:4]) + list(below[:3]):
+        assert oracle_mod.pair_t(float(x1[i]), float(x2[i])) == t[i]
+        begin = max(int(i) - (1 << 20), 0)
+        g = gpu_range(env, NPB_SEED, NPB_A, begin, 1 << 21)
+        assert_parity(g, oracle_mod.run_pairs(NPB_SEED, NPB_A, begin, 1 << 21))

@@ -33,7 +33,9 @@ for addr, i in ins:
     if m and int(m.group(1), 16) < addr:
         lo = int(m.group(1), 16)
         n = sum(1 for a, j in ins if lo <= a <= addr and "RSQ64H" in j)
-        if best is None or n > best[2] or (n == best[2] and addr - lo < best[1] - best[0]):
+        # the pipelined group loop holds exactly one MUFU per pair of an
+        # iteration (ppi); among such loops take the smallest
+        if n == ppi and (best is None or addr - lo < best[1] - best[0]):
             best = (lo, addr, n)
 lo, hi, _ = best
 body = [(a, i) for a, i in ins if lo <= a <= hi]
