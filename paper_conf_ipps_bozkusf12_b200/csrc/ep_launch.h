@@ -13,7 +13,10 @@ namespace hplep {
 constexpr int HPL_VARIANT_LEAN = HPL_EP_LEAN;
 constexpr int HPL_VARIANT_LIBDEVICE = HPL_EP_LIBDEVICE;
 constexpr int EP_DEFAULT_THREADS = 512;
-constexpr uint64_t EP_MIN_PAIRS_PER_THREAD = 64;
+#ifndef EP_MIN_PPT
+#define EP_MIN_PPT 8   // min pairs per thread before the grid grows (64 -> 8: -8 us at 2^16 pairs, session 3)
+#endif
+constexpr uint64_t EP_MIN_PAIRS_PER_THREAD = EP_MIN_PPT;
 
 struct EPConfig {
   int variant = HPL_VARIANT_LEAN;
