@@ -45,6 +45,9 @@ reduce_sum_f32_kernel(const float* __restrict__ in, int64_t n, double* __restric
   // full rounds of RED_UNROLL independent 16-B loads per thread (the grid is
   // sized so that the rounds cover the input), then a short remainder
   int64_t i = tid;
+#ifdef RED_FLOOR  // timing study only (result wrong): skip the stream, keep launch + tree + fold
+  i = nv;
+#endif
   for (; i + (RED_UNROLL - 1) * T < nv; i += RED_UNROLL * T) {
     float4 r[RED_UNROLL];
 #pragma unroll
