@@ -1,7 +1,9 @@
 /* A plain C client of the C ABI (include/hpl.h) — no Python, no torch.
  *   cpu  : library loads, status strings, argument validation (no GPU needed)
  *   gpu  : NPB class S through hpl_ep_run and the Array/eval path, checked
- *          against NPB's published verification sums (tests/golden) */
+ *          against NPB's published verification sums (tests/golden); the
+ *          transpose through eval on Arrays and the reduction on an Array's
+ *          device copy, checked against their definitions */
 #include <math.h>
 #include <stdio.h>
 #include <string.h>
@@ -25,6 +27,9 @@ int main(int argc, char** argv) {
   CHECK(strlen(hpl_last_error()) > 0);
   CHECK(hpl_ep_run_shard(24, 271828183ull, 1220703125ull, 3, 2, (double*)0x1000, NULL) == HPL_EINVAL);
   CHECK(hpl_eval("no_such_kernel", 0, NULL, NULL, 0, NULL) == HPL_EINVAL);
+  CHECK(hpl_transpose_f32(NULL, 0, 7, NULL, NULL) == HPL_OK);                       /* empty */
+  CHECK(hpl_transpose_f32((const float*)0x1000, 3, 4, (float*)0x1008, NULL) == HPL_EINVAL);  /* overlap */
+  CHECK(hpl_reduce_sum_f32(NULL, -1, (double*)0x1000, NULL) == HPL_EINVAL);
   if (gpu) {
     /* NPB class S (M = 24); verification values: NPB ep.f (BASELINE.json) */
     CHECK(hpl_ep_run(24, 271828183ull, 1220703125ull, &sx, &sy, q) == HPL_OK);
@@ -45,6 +50,45 @@ int main(int argc, char** argv) {
     CHECK(hpl_array_data(out, HPL_HOST, (void**)&h) == HPL_OK);
     CHECK(h[0] == sx && h[1] == sy && (uint64_t)h[12] == gc);
     CHECK(hpl_array_free(out) == HPL_OK);
+
+    /* transpose (Fig. 10(b)) through eval on two Arrays: dest (w x h) = src (h x w) */
+    enum { H = 70, W = 131 };
+    hpl_array src, dst;
+    int64_t ds[2] = {H, W}, dd[2] = {W, H};
+    CHECK(hpl_array_alloc(&src, HPL_F32, 2, ds, NULL, -1) == HPL_OK);
+    CHECK(hpl_array_alloc(&dst, HPL_F32, 2, dd, NULL, -1) == HPL_OK);
+    float* hs;
+    CHECK(hpl_array_data(src, HPL_HOST, (void**)&hs) == HPL_OK);
+    for (int i = 0; i < H * W; ++i) hs[i] = (float)i * 0.5f - 100.0f;
+    CHECK(hpl_array_sync(src, HPL_HOST, HPL_WRITE) == HPL_OK);
+    hpl_arg args[2];
+    memset(args, 0, sizeof(args));
+    args[0].kind = HPL_ARG_ARRAY; args[0].array = dst;
+    args[1].kind = HPL_ARG_ARRAY; args[1].array = src;
+    CHECK(hpl_eval("transpose_f32", 0, NULL, NULL, 2, args) == HPL_OK);
+    CHECK(hpl_array_sync(dst, HPL_HOST, HPL_READ) == HPL_OK);
+    float* hd;
+    CHECK(hpl_array_data(dst, HPL_HOST, (void**)&hd) == HPL_OK);
+    int bad = 0;
+    for (int i = 0; i < H; ++i)
+      for (int j = 0; j < W; ++j) bad += hd[j * H + i] != hs[i * W + j];
+    CHECK(bad == 0);
+    /* reduction of src's device copy: sum of (i/2 - 100), exact in double */
+    void* dsrc;
+    double* dsum;
+    hpl_array sum;
+    int64_t one = 1;
+    CHECK(hpl_array_alloc(&sum, HPL_F64, 1, &one, NULL, -1) == HPL_OK);
+    CHECK(hpl_array_data(src, HPL_DEVICE, &dsrc) == HPL_OK);
+    CHECK(hpl_array_data(sum, HPL_DEVICE, (void**)&dsum) == HPL_OK);
+    CHECK(hpl_reduce_sum_f32((const float*)dsrc, H * W, dsum, NULL) == HPL_OK);
+    CHECK(hpl_array_sync(sum, HPL_DEVICE, HPL_WRITE) == HPL_OK);  /* the kernel wrote the device copy */
+    CHECK(hpl_array_sync(sum, HPL_HOST, HPL_READ) == HPL_OK);
+    double* hsum;
+    CHECK(hpl_array_data(sum, HPL_HOST, (void**)&hsum) == HPL_OK);
+    const double n = (double)(H * W), want = 0.5 * n * (n - 1) / 2.0 - 100.0 * n;
+    CHECK(*hsum == want);
+    CHECK(hpl_array_free(src) == HPL_OK && hpl_array_free(dst) == HPL_OK && hpl_array_free(sum) == HPL_OK);
   }
   printf("%s: %d failures\n", gpu ? "gpu" : "cpu", fails);
   return fails != 0;
