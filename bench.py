@@ -167,9 +167,62 @@ def run_reference(args, M):
     return 0
 
 
-def cpu_baseline_sample(M, budget_s):
-    """Oracle as it stands on the host cores over a bounded sample of class M."""
+def verify_result(cls, M, result, world):
+    """Correctness gate of the measured run: the
+    printed result against NPB's published verification sums (relative 1e-8,
+    ep.f's epsilon) and, where a stored oracle result exists for the class
+    (tests/golden/oracle_ep.json, written by a script that calls only oracle/;
+    or NPB's reference counts for S/W/A), q[] and gc exactly and sx, sy within
+    T1 = 1e-12 * max(|ref|, sqrt(gc)).  Returns the "verified" record."""
+    gdir = os.path.join(ROOT, "tests", "golden")
+    checks, ok = [], True
+    sx, sy, q, gc = result["sx"], result["sy"], result["q"], result["gc"]
+    if not (sx == sx and sy == sy) or sum(q) != gc:
+        return {"ok": False, "checks": ["result is NaN or sum(q) != gc (combine failed?)"]}
+    for line in open(os.path.join(gdir, "npb_ep_verify.txt")):
+        f = line.split()
+        if f and not f[0].startswith("#") and f[0] == cls:
+            good = abs((sx - float(f[2])) / float(f[2])) <= 1e-8 and abs((sy - float(f[3])) / float(f[3])) <= 1e-8
+            checks.append("NPB verification sums (1e-8): %s" % ("pass" if good else "FAIL"))
+            ok &= good
+    gold = json.load(open(os.path.join(gdir, "oracle_ep.json"))).get(cls)
+    if gold is not None:
+        rs, ry = float.fromhex(gold["sx"]), float.fromhex(gold["sy"])
+        tol = 1e-12 * max(abs(rs), abs(ry), gold["gc"] ** 0.5)
+        good = q == gold["q"] and gc == gold["gc"]
+        checks.append("q, gc exact vs oracle golden: %s" % ("pass" if good else "FAIL"))
+        ok &= good
+        good = abs(sx - rs) <= 1e-12 * max(abs(rs), gold["gc"] ** 0.5) and \
+            abs(sy - ry) <= 1e-12 * max(abs(ry), gold["gc"] ** 0.5)
+        checks.append("sx, sy within 1e-12*max(|ref|, sqrt(gc)) of oracle golden: %s (|d| %.2e, %.2e; tol %.2e)"
+                      % ("pass" if good else "FAIL", abs(sx - rs), abs(sy - ry), tol))
+        ok &= good
+    else:
+        for line in open(os.path.join(gdir, "npb_ep_counts.txt")):
+            f = line.split()
+            if f and not f[0].startswith("#") and f[0] == cls:
+                good = gc == int(f[2]) and q[:7] == [int(v) for v in f[3:10]]
+                checks.append("q, gc exact vs NPB reference counts: %s" % ("pass" if good else "FAIL"))
+                ok &= good
+    if not checks:
+        checks.append("no stored reference for class %s" % cls)
+    return {"ok": bool(ok), "world": world, "checks": checks}
+
+
+def cpu_baseline_sample(M, budget_s, single_s=6.0):
+    """Oracle as it stands on the host cores over a bounded sample of class M,
+    and (the paper's serial-CPU baseline) the
+    same oracle on ONE core over a smaller sample."""
     import oracle
+    t0 = time.perf_counter()
+    oracle.run_batches(M, NPB_SEED, NPB_A, 0, 1, threads=1, margin=False)
+    t_b = max(time.perf_counter() - t0, 1e-3)
+    nb1 = max(1, min(int(single_s / t_b), 1 << (M - 16)))
+    t0 = time.perf_counter()
+    oracle.run_batches(M, NPB_SEED, NPB_A, 0, nb1, threads=1, margin=False)
+    dt1 = time.perf_counter() - t0
+    single = {"value": round(2 * (nb1 << 16) / dt1 / 1e6, 3), "unit": UNIT, "cores": 1,
+              "sample": "first %d NPB batches (%d pairs, %.1f s), one thread" % (nb1, nb1 << 16, dt1)}
     threads = os.cpu_count() or 1
     t0 = time.perf_counter()
     oracle.run_batches(M, NPB_SEED, NPB_A, 0, threads, threads=threads, margin=False)
@@ -182,7 +235,8 @@ def cpu_baseline_sample(M, budget_s):
     pairs = batches << 16
     return {"value": round(2 * pairs / dt / 1e6, 3), "unit": UNIT, "cores": threads, "kind": "oracle",
             "sample": "first %d NPB batches of class-%d stream (%d pairs, %.1f s), batch-parallel over "
-                      "%d threads, margin tracking off" % (batches, M, pairs, dt, threads)}
+                      "%d threads, margin tracking off" % (batches, M, pairs, dt, threads),
+            "single_core": single}
 
 
 # --------------------------------------------------------------------- ours
@@ -267,6 +321,16 @@ def run_ours(args, M):
         dist.barrier()
     clocks = sampler.stop()
     result = hpl.unpack13(out.cpu().tolist())
+    combine_failures = 0
+    if combine == "fused":
+        try:
+            fc.status()  # every timed combine completed (no timeout / torn slot)
+        except hpl.HPLError:
+            combine_failures = 1
+    verified = verify_result(args.cls, M, result, world)
+    if combine_failures:
+        verified["ok"] = False
+        verified["checks"].append("fused combine reported a failed call")
 
     total_ms = sum(step_ms)
     t = torch.tensor([total_ms, sum(kern_ms), float(launches)], dtype=torch.float64, device=dev)
@@ -300,6 +364,14 @@ def run_ours(args, M):
             multi.ep_run_distributed(M, NPB_SEED, NPB_A, device=dev)
         e2e_ms.append((time.perf_counter() - t0) * 1e3)
     e2e_tot = sum(e2e_ms)
+    if combine == "fused":
+        fc.status()
+    if world == 1:
+        e2e_res = {"sx": sx, "sy": sy, "q": q, "gc": sum(q)}
+        v2 = verify_result(args.cls, M, e2e_res, world)
+        if not v2["ok"]:
+            verified["ok"] = False
+            verified["checks"].append("e2e (hpl_ep_run) result: " + "; ".join(v2["checks"]))
     if world > 1:
         te = torch.tensor([e2e_tot], dtype=torch.float64, device=dev)
         dist.all_reduce(te, op=dist.ReduceOp.MAX)
@@ -317,8 +389,12 @@ def run_ours(args, M):
         kern_avg_s = kern_max_ms / args.steps / 1e3
         achieved = ALG_OPS_PER_PAIR * pairs_per_launch / kern_avg_s
         traffic = load_profile_traffic()
+        per_step = sorted(units / (ms / 1e3) / 1e6 for ms in step_ms)  # rank 0's steps
         line = {
             "metric": METRIC, "value": round(value, 1), "unit": UNIT, "n_gpus": world,
+            "value_stats": {"median": round(statistics.median(per_step), 1), "min": round(per_step[0], 1),
+                            "max": round(per_step[-1], 1), "steps": len(per_step),
+                            "note": "per-step Mops/s (rank 0); value = all steps / their total time"},
             "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": round(total_ms / args.steps, 4), "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "f64",
@@ -351,16 +427,23 @@ def run_ours(args, M):
             "gpu_launches": launches_all,
             "clocks": clocks,
             "dist_backend": args.dist_backend if world > 1 else None,
-            "result": {"sx": result["sx"], "sy": result["sy"], "gc": result["gc"]},
+            "result": {"sx": result["sx"], "sy": result["sy"], "gc": result["gc"], "q": result["q"]},
+            "verified": verified["ok"],
+            "verification": verified["checks"],
         }
         if not args.no_cpu_baseline and world == 1:
             line["cpu_baseline"] = cpu_baseline_sample(M, args.cpu_budget)
         print(json.dumps(line), flush=True)
     if fc is not None:
         fc.close()
+    ok = torch.tensor([1.0 if verified["ok"] else 0.0], dtype=torch.float64, device=dev)
     if world > 1:
+        dist.all_reduce(ok, op=dist.ReduceOp.MIN)
         dist.barrier()
         dist.destroy_process_group()
+    if ok.item() != 1.0:
+        sys.stderr.write("bench: result verification FAILED: %s\n" % "; ".join(verified["checks"]))
+        return 3
     return 0
 
 

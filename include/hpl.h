@@ -34,6 +34,7 @@
 #ifndef HPL_H_
 #define HPL_H_
 
+#include <stddef.h>
 #include <stdint.h>
 
 #ifdef __cplusplus
@@ -56,6 +57,27 @@ const char* hpl_strerror(int code);
 const char* hpl_last_error(void);
 /* Library ABI version: (major << 16) | minor. */
 int hpl_version(void);
+
+/* ---- device memory and library state ----------------------------------
+ * Device memory the library allocates for the caller (hpl_array device
+ * copies, the temporary buffers of the test hooks) comes from cudaMalloc
+ * unless an allocator is installed: alloc(bytes, device, ctx) returns device
+ * memory on `device` (NULL = out of memory, reported as HPL_ENOMEM) and
+ * free(ptr, bytes, device, ctx) releases it.  The Python binding installs
+ * torch's caching allocator, so arrays share the pool of the caller's tensors
+ * (reading B1).  An array is always freed with the
+ * allocator that allocated it.  alloc and free must both be NULL (restore
+ * cudaMalloc) or both non-NULL.  Internal per-device state (the EP log table,
+ * reduction workspaces) stays on cudaMalloc and is released by hpl_shutdown. */
+typedef void* (*hpl_alloc_fn)(size_t bytes, int device, void* ctx);
+typedef void (*hpl_free_fn)(void* ptr, size_t bytes, int device, void* ctx);
+int hpl_set_device_allocator(hpl_alloc_fn alloc, hpl_free_fn free_fn, void* ctx);
+/* Release every library-owned buffer: the calling thread's hpl_ep_run result
+ * arrays (other threads' are freed at their exit), the EP log tables and
+ * workspaces and the reduction workspaces of every device (each synchronised
+ * first), and restore the cudaMalloc allocator.  Call with no library work
+ * pending; the next call re-creates what it needs. */
+int hpl_shutdown(void);
 
 /* ---- devices ----------------------------------------------------------- */
 int hpl_device_count(int* n);
@@ -137,7 +159,8 @@ int hpl_ep_run_range(uint64_t seed, uint64_t a, uint64_t pair_begin, uint64_t np
 
 /* Test hook: the LCG states x_{offset+1} .. x_{offset+n} (u64 < 2^46),
  * computed on the device by the same skip-ahead and step code the EP kernel
- * uses, copied to host_out[0..n-1].  Blocking.  n <= 2^28. */
+ * uses (its skip-ahead and the hot loop's step function), copied to
+ * host_out[0..n-1].  Blocking.  n <= 2^28. */
 int hpl_lcg_states(uint64_t seed, uint64_t a, uint64_t offset, uint64_t n, uint64_t* host_out);
 
 /* ---- fused cross-GPU combine ----------------------------
@@ -146,10 +169,13 @@ int hpl_lcg_states(uint64_t seed, uint64_t a, uint64_t offset, uint64_t n, uint6
  * §8(e)).  Instead of a separate allreduce, hpl_ep_run_fused's kernel does
  * it itself: its last block stores the shard's partial into slot [rank] of
  * every rank's inbox (device memory of that rank's GPU, mapped into this
- * process with CUDA IPC; peer stores over NVLink), signals each inbox with a
- * system-scope release add, waits (acquire) until its own inbox holds all
- * nranks partials of this call, and sums them in rank order into dev_out13.
- * Every rank therefore ends with the same, bitwise reproducible result.
+ * process with CUDA IPC; peer stores over NVLink), then a tag word holding
+ * the call's epoch with a system-scope release; it waits (acquire) until
+ * every slot of its own inbox carries this call's epoch, sums the nranks
+ * partials in rank order into dev_out13 and re-checks the tags (a peer that
+ * gave up waiting and moved on would have changed them: the call then
+ * reports failure instead of mixing calls).  Every rank therefore ends with
+ * the same, bitwise reproducible result.
  * Setup, one process per GPU (or several processes sharing one GPU):
  *   1. hpl_comm_create(&c, rank, nranks, device, handle) on every rank;
  *   2. exchange the HPL_COMM_HANDLE_BYTES handles (e.g. an all_gather over
@@ -161,7 +187,8 @@ int hpl_lcg_states(uint64_t seed, uint64_t a, uint64_t offset, uint64_t n, uint6
 #define HPL_COMM_HANDLE_BYTES 64
 #define HPL_COMM_MAX_RANKS 8
 typedef struct hpl_comm_s* hpl_comm;
-/* nranks in [1, 8], 0 <= rank < nranks; device -1 = current.  Writes the
+/* nranks a power of two in [1, 8] (equal shards), 0 <= rank < nranks;
+ * device -1 = current.  Writes the
  * 64-byte IPC handle of this rank's inbox to handle_out. */
 int hpl_comm_create(hpl_comm* out, int rank, int nranks, int device, void* handle_out);
 /* Map the peers' inboxes (handles in rank order; this rank's own entry is
@@ -176,7 +203,9 @@ int hpl_comm_free(hpl_comm c);
  * problem's result on every rank.  Asynchronous on `stream`. */
 int hpl_ep_run_fused(hpl_comm c, int M, uint64_t seed, uint64_t a, double* dev_out13, void* stream);
 /* Synchronize `stream`; report the number of fused calls issued (epoch) and
- * of calls whose combine timed out.  Returns HPL_ECUDA if timeouts > 0. */
+ * of calls whose combine failed (timed out waiting for a peer, or saw a
+ * peer's slot change during the fold; word 0 of those results is NaN).
+ * Returns HPL_ECUDA if any failed. */
 int hpl_comm_status(hpl_comm c, void* stream, uint64_t* epoch, uint64_t* timeouts);
 
 /* ---- reduction -----------------------------------------

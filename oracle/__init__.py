@@ -80,6 +80,12 @@ def _load():
         lib.ep_oracle_run.restype = i
         lib.ep_oracle_run_pairs.argtypes = [d, d, u64, u64, i, R]
         lib.ep_oracle_run_pairs.restype = i
+        lib.ep_oracle_csum.argtypes = [ctypes.c_void_p, u64]
+        lib.ep_oracle_csum.restype = d
+        lib.ep_oracle_bin_margin.argtypes = [d]
+        lib.ep_oracle_bin_margin.restype = d
+        lib.ep_oracle_pairs.argtypes = [d, d, u64, u64, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p]
+        lib.ep_oracle_pairs.restype = i
         _lib = lib
     return _lib
 
@@ -144,3 +150,24 @@ def run_pairs(seed: int, a: int, p_begin: int, npairs: int, margin: bool = True)
     rc = _load().ep_oracle_run_pairs(float(seed), float(a), p_begin, npairs, int(margin),
                                      ctypes.byref(r))
     return _conv(r, rc)
+
+
+def csum(values) -> float:
+    """The oracle's Neumaier-compensated sum (reading R10) of a float sequence."""
+    import numpy as np
+    v = np.ascontiguousarray(values, dtype=np.float64)
+    return _load().ep_oracle_csum(v.ctypes.data, v.size)
+
+
+def bin_margin(m: float) -> float:
+    """Reading R7: ulps from m to the nearest integer in 1..10 (1e300 if none)."""
+    return _load().ep_oracle_bin_margin(m)
+
+
+def pairs(seed: int, a: int, p_begin: int, n: int):
+    """Per-pair deviates (X, Y, l) of pairs [p_begin, p_begin + n) as numpy
+    arrays; rejected pairs have X = Y = 0 and l = -1."""
+    import numpy as np
+    X = np.zeros(max(n, 1)); Y = np.zeros(max(n, 1)); l = np.zeros(max(n, 1), dtype=np.int64)
+    _load().ep_oracle_pairs(float(seed), float(a), p_begin, n, X.ctypes.data, Y.ctypes.data, l.ctypes.data)
+    return X[:n], Y[:n], l[:n]

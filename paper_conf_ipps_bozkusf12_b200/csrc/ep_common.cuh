@@ -65,6 +65,22 @@ constexpr uint32_t LOG_ADD = (uint32_t(1) << (LOG_SHIFT - 1)) - (LOG_IDX_MIN << 
 constexpr uint32_t LOG_TINY = LOG_N + 512;
 constexpr uint32_t LOG_TAB = LOG_TINY + 1;
 
+// Truncating index (EP_IDX_TRUNC=1, the default): entry j of the table holds
+// the bucket of every t' whose high word H has H >> LOG_SHIFT == j + TRUNC_J0,
+// i.e. [lo_j, lo_j + w) with the reference point at its centre (so |r| has the
+// same bound as with round-to-nearest buckets).  Entry 0 (j0 = IDX_MIN - 1) is
+// the "below the table" sentinel {T = 60, inv = 0}, reached through the clamp
+// max(H, TRUNC_HLO); the two buckets around t' = 1/4 ([1/4 - w, 1/4) and
+// [1/4, 1/4 + w)) take 1/4 itself as reference point (inv = 4, T = 0, r exact),
+// so L = -2 ln(1 + r) never cancels against T as t' -> 1/4; t' = 1/4 gives
+// L = 0 (X = Y = 0, bin 0) and every t' > 1/4 a negative L (NaN -> rare path
+// -> exact reject); the entries above are reject sentinels up to t' = 1/2.  Address = ((max(H, HLO) >> 11) << 4) + base':
+// VIMNMX + SHF + LEA, no recentring add.
+constexpr uint32_t TRUNC_J0 = LOG_IDX_MIN - 1;
+constexpr uint32_t TRUNC_HLO = TRUNC_J0 << LOG_SHIFT;
+constexpr uint32_t TRUNC_TAB = ((LOG_BIAS_TOP + 1) << LOG_K) - TRUNC_J0 + 1;  // up to t' = 1/2
+static_assert(TRUNC_TAB == LOG_TAB, "same table footprint in both index modes");
+
 struct LogEntry {
   double T;    // RN(2 ln(inv / 4))
   double inv;  // float-representable ~1/centre
@@ -80,12 +96,14 @@ struct EPPartial {
 // ---- fused cross-GPU combine ---------------------------
 // Every rank owns one CommInbox in its own device memory; peers write into it
 // over NVLink (CUDA IPC mappings).  slot[epoch & 1][r] holds rank r's 13-word
-// partial {sx, sy, q0..q9, big}; `arrived` counts partials (system-scope
-// atomic adds, monotonic over calls: after call e it is e * nranks).
+// partial {sx, sy, q0..q9, big} in words 0..12 and, in word COMM_TAG, the
+// epoch (1, 2, ... per fused call) of the call that wrote it, stored with a
+// system-scope release after the data.
 constexpr int COMM_MAX_RANKS = 8;
+constexpr int COMM_TAG = 13;
 struct CommInbox {
   double slot[2][COMM_MAX_RANKS][16];
-  unsigned long long arrived;
+  unsigned long long stale;     // calls whose tags changed during the fold (a peer ran ahead)
   unsigned long long timeouts;  // calls whose wait gave up (peer missing)
 };
 struct CommParams {

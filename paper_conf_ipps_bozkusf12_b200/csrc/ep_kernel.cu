@@ -26,6 +26,7 @@
 namespace hplep {
 
 constexpr int EP_MAX_THREADS = 1024;
+constexpr int EP_MAX_BLOCKS_PER_SM = 32;  // hpl_ep_set_config's blocks_per_sm bound (hardware limit)
 
 __device__ __forceinline__ double as_double(uint64_t v) {
   return __longlong_as_double(static_cast<long long>(v));
@@ -43,6 +44,34 @@ __device__ __forceinline__ double rsqrt_approx(double p) {
   double y;
   asm("rsqrt.approx.ftz.f64 %0, %1;" : "=d"(y) : "d"(p));  // MUFU.RSQ64H, ~2^-20
   return y;
+}
+
+#ifndef EP_IDX_TRUNC
+#define EP_IDX_TRUNC 1  // 1: truncating table index (VIMNMX + SHF + LEA; ep_common.cuh)
+#endif
+#ifndef EP_LCG_CARRY
+#define EP_LCG_CARRY 1  // 1: LCG carries the unmasked high word (IMAD reads one odd register)
+#endif
+#ifndef EP_E_SQ
+#define EP_E_SQ 1       // 1: Newton residual e = 1 - p y0^2 with y0^2 exact (one register pair)
+#endif
+
+// Shared-memory address of the log-table entry of t' (high word H).  `tabb` is
+// the table base, pre-biased by -TRUNC_J0 entries in the truncating mode.
+__device__ __forceinline__ unsigned tab_addr(unsigned H, unsigned tabb) {
+#if EP_IDX_TRUNC
+  return ((max(H, TRUNC_HLO) >> LOG_SHIFT) << 4) + tabb;
+#else
+  return (min((H + LOG_ADD) >> LOG_SHIFT, LOG_N) << 4) + tabb;
+#endif
+}
+__device__ __forceinline__ unsigned tab_base(const void* smem) {
+  const unsigned b = static_cast<unsigned>(__cvta_generic_to_shared(smem));
+  return EP_IDX_TRUNC ? b - TRUNC_J0 * 16u : b;
+}
+// t' below the table (truncating mode; the exact rare path recomputes these pairs)
+__device__ __forceinline__ bool below_table(double t) {
+  return static_cast<unsigned>(__double2hiint(t)) < (LOG_IDX_MIN << LOG_SHIFT);
 }
 
 #ifndef EP_Y0LO
@@ -126,6 +155,19 @@ __device__ __forceinline__ void lcg_step_k(unsigned& lo, unsigned& hi, unsigned 
   asm("lop3.b32 %0, %1, 0x000FFFFF, %2, 0xEA;" : "=r"(hi) : "r"(ph), "r"(exp_hi));
 }
 
+// Same step carrying the UNMASKED high word ph: a * (bits above 2^52) only
+// reaches bits >= 2^52 of the product, so ph' = hi(a v) + a ph agrees with the
+// masked recurrence on bits 0..19; the double's high word hd is the masked copy.
+// The IMAD then reads ph (any register parity) and the odd carry word instead
+// of two odd registers (RF-bank conflict).
+template <bool A32>
+__device__ __forceinline__ void lcg_step_c(unsigned& lo, unsigned& ph, unsigned& hd, unsigned a_lo, unsigned a_hi,
+                                           unsigned exp_hi) {
+  ph = __umulhi(lo, a_lo) + ph * a_lo + (A32 ? 0u : lo * a_hi);
+  lo = lo * a_lo;
+  asm("lop3.b32 %0, %1, 0x000FFFFF, %2, 0xEA;" : "=r"(hd) : "r"(ph), "r"(exp_hi));
+}
+
 template <bool A32>
 __device__ __forceinline__ void lcg_step(unsigned& lo, unsigned& hi, unsigned a_lo, unsigned a_hi) {
   const unsigned ph = __umulhi(lo, a_lo) + hi * a_lo + (A32 ? 0u : lo * a_hi);
@@ -178,8 +220,13 @@ struct RareOut {
 __device__ __noinline__ RareOut rare_pair(double t, double x1, double x2, double X, double Y,
                                           unsigned u, unsigned long long* s_rare) {
   if (t > 0.25) return RareOut{0.0, 0.0, 0u};  // rejected (never routed here by the fast path)
+#if EP_IDX_TRUNC
+  (void)u;
+  if (below_table(t)) {
+#else
   if (u == ~0u) u = (static_cast<unsigned>(__double2hiint(t)) + LOG_ADD) >> LOG_SHIFT;  // wraps below the table
-  if (u >= LOG_N) {  // t below the table: NPB's formula, libdevice log/sqrt, on
+  if (u >= LOG_N) {
+#endif  // t below the table: NPB's formula, libdevice log/sqrt, on
     // the unscaled t = 4 t', x = 2 x' (exact)
     const double tt = 4.0 * t;
     const double t2 = sqrt(-2.0 * log(tt) / tt);
@@ -213,9 +260,9 @@ __device__ __forceinline__ void lean_pair(unsigned& vlo, unsigned& vhi, const EP
   const bool acc = t <= 0.25;
   // A5: L = -2 ln(4 t) from the table entry of t (sentinel for t outside)
   const unsigned H = static_cast<unsigned>(__double2hiint(t));
-  const unsigned u = min((H + LOG_ADD) >> LOG_SHIFT, LOG_N);
+  const unsigned u = min((H + LOG_ADD) >> LOG_SHIFT, LOG_N);  // (only the rounding mode's rare path reads it)
   double eT, eInv;
-  asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(eT), "=d"(eInv) : "r"((u << 4) + tab));
+  asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(eT), "=d"(eInv) : "r"(tab_addr(H, tab)));
   const double r = fma(t, eInv, -1.0);
   double c = fma(r, EP_C6, EP_C5);
   c = fma(c, r, 0.5);
@@ -226,8 +273,7 @@ __device__ __forceinline__ void lean_pair(unsigned& vlo, unsigned& vhi, const EP
   // t2' = sqrt(L/t) = L rsqrt(L t): MUFU seed + one cubic Newton step
   const double p = fma(L, t, 0x1p-200);  // + 2^-200: t' == 1/4 -> L = 0 -> t2' = 0
   const double y0 = rsqrt_approx(p);
-  const double h = __dmul_rn(p, y0);
-  const double e = fma(-h, y0, 1.0);
+  const double e = EP_E_SQ ? fma(-p, __dmul_rn(y0, y0), 1.0) : fma(-__dmul_rn(p, y0), y0, 1.0);
   const double cc = fma(e, 0.375, 0.5);
   const double g = __dmul_rn(L, y0);
   const double ge = __dmul_rn(g, e);
@@ -243,7 +289,7 @@ __device__ __forceinline__ void lean_pair(unsigned& vlo, unsigned& vhi, const EP
     A.cnt += bin_increment(l);
   }
   if (acc && !ok) {
-    const RareOut o = rare_pair(t, x1, x2, X, Y, u, s_rare);
+    const RareOut o = rare_pair(t, x1, x2, X, Y, EP_IDX_TRUNC ? ~0u : u, s_rare);
     A.csx += o.dx;
     A.csy += o.dy;
     A.cnt += o.dcnt;
@@ -306,7 +352,8 @@ __device__ __forceinline__ void lean_pairs(unsigned& vlo, unsigned& vhi, const E
   double eT[W], eInv[W];
 #pragma unroll
   for (int k = 0; k < W; ++k)
-    asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(eT[k]), "=d"(eInv[k]) : "r"((u[k] << 4) + tab));
+    asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(eT[k]), "=d"(eInv[k])
+                 : "r"(tab_addr(static_cast<unsigned>(__double2hiint(t[k])), tab)));
   double r[W], c[W], L[W];
 #pragma unroll
   for (int k = 0; k < W; ++k) {
@@ -330,7 +377,8 @@ __device__ __forceinline__ void lean_pairs(unsigned& vlo, unsigned& vhi, const E
     y0[k] = rsqrt_approx(p[k]);
   }
 #pragma unroll
-  for (int k = 0; k < W; ++k) e[k] = fma(-__dmul_rn(p[k], y0[k]), y0[k], 1.0);
+  for (int k = 0; k < W; ++k)
+    e[k] = EP_E_SQ ? fma(-p[k], __dmul_rn(y0[k], y0[k]), 1.0) : fma(-__dmul_rn(p[k], y0[k]), y0[k], 1.0);
 #pragma unroll
   for (int k = 0; k < W; ++k) {
     g[k] = __dmul_rn(L[k], y0[k]);
@@ -354,7 +402,7 @@ __device__ __forceinline__ void lean_pairs(unsigned& vlo, unsigned& vhi, const E
 #pragma unroll
     for (int k = 0; k < W; ++k)
       if (acc[k] && !ok[k]) {
-        const RareOut o = rare_pair(t[k], x1[k], x2[k], X[k], Y[k], u[k], s_rare);
+        const RareOut o = rare_pair(t[k], x1[k], x2[k], X[k], Y[k], EP_IDX_TRUNC ? ~0u : u[k], s_rare);
         A.csx += o.dx;
         A.csy += o.dy;
         A.cnt += o.dcnt;
@@ -428,16 +476,27 @@ __device__ __forceinline__ void gen_stage(unsigned& vlo, unsigned& vhi, const EP
   for (int k = 0; k < W; ++k) {
 #if EP_ABL & 2  // ablation (timing only, wrong results): LCG step -> one add
     vlo += P.a_lo;
+#elif EP_LCG_CARRY
+    unsigned hd;  // vhi carries the unmasked high word (lcg_step_c)
+    lcg_step_c<A32>(vlo, vhi, hd, P.a_lo, P.a_hi, exp_hi);
+    S.x1[k] = __dadd_rn(__hiloint2double(int(hd), int(vlo)), -1.5);
 #else
     lcg_step_k<A32>(vlo, vhi, P.a_lo, P.a_hi, exp_hi);
 #endif
+#if !EP_LCG_CARRY || (EP_ABL & 2)
     S.x1[k] = __dadd_rn(__hiloint2double(int(vhi), int(vlo)), -1.5);
+#endif
 #if EP_ABL & 2
     vhi ^= vlo;
+#elif EP_LCG_CARRY
+    lcg_step_c<A32>(vlo, vhi, hd, P.a_lo, P.a_hi, exp_hi);
+    S.x2[k] = __dadd_rn(__hiloint2double(int(hd), int(vlo)), -1.5);
 #else
     lcg_step_k<A32>(vlo, vhi, P.a_lo, P.a_hi, exp_hi);
 #endif
+#if !EP_LCG_CARRY || (EP_ABL & 2)
     S.x2[k] = __dadd_rn(__hiloint2double(int(vhi), int(vlo)), -1.5);
+#endif
   }
 #pragma unroll
   for (int k = 0; k < W; ++k) {
@@ -448,7 +507,9 @@ __device__ __forceinline__ void gen_stage(unsigned& vlo, unsigned& vhi, const EP
 #else
     S.t[k] = __dadd_rn(__dmul_rn(S.x1[k], S.x1[k]), __dmul_rn(S.x2[k], S.x2[k]));
 #endif
-#if EP_IDX_FUSED
+#if EP_IDX_TRUNC
+    // (no stage index: the rare path tests below_table(t) itself)
+#elif EP_IDX_FUSED
     // clamp before the shift (same index; lets ptxas fuse add + min: VIADDMNMX)
     constexpr unsigned LIM = ((EP_PRED_MODE == 1 ? LOG_TINY : LOG_N) << LOG_SHIFT) | ((1u << LOG_SHIFT) - 1);
     S.u[k] = min(static_cast<unsigned>(__double2hiint(S.t[k])) + LOG_ADD, LIM) >> LOG_SHIFT;
@@ -462,6 +523,9 @@ __device__ __forceinline__ void gen_stage(unsigned& vlo, unsigned& vhi, const EP
 #if EP_ABL & 1  // ablation: no table lookup / index
     S.eT[k] = S.x1[k];
     S.eInv[k] = S.x2[k];
+#elif EP_IDX_TRUNC
+    asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(S.eT[k]), "=d"(S.eInv[k])
+                 : "r"(tab_addr(static_cast<unsigned>(__double2hiint(S.t[k])), tab)));
 #else
     asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(S.eT[k]), "=d"(S.eInv[k]) : "r"((S.u[k] << 4) + tab));
 #endif
@@ -522,14 +586,15 @@ __device__ __forceinline__ void transform_stage(const Stage<W>& S, const EPParam
     y0[k] = rsqrt_approx(p[k]);
 #endif
   }
-#if EP_Y0LO
+#if EP_Y0LO && !EP_E_SQ
   // e = 1 - p y0^2 as 1 - (L y0)(t y0): p is dead after the MUFU (its
   // register pair can hold y0), g = L y0 is reused below
 #pragma unroll
   for (int k = 0; k < W; ++k) e[k] = fma(-__dmul_rn(L[k], y0[k]), __dmul_rn(S.t[k], y0[k]), 1.0);
 #else
 #pragma unroll
-  for (int k = 0; k < W; ++k) e[k] = fma(-__dmul_rn(p[k], y0[k]), y0[k], 1.0);
+  for (int k = 0; k < W; ++k)
+    e[k] = EP_E_SQ ? fma(-p[k], __dmul_rn(y0[k], y0[k]), 1.0) : fma(-__dmul_rn(p[k], y0[k]), y0[k], 1.0);
 #endif
   bool any_rare = false;
   unsigned sel_min = 0xFFFFFFFFu;
@@ -614,7 +679,7 @@ __device__ __forceinline__ void transform_stage(const Stage<W>& S, const EPParam
           X[k] = __dmul_rn(S.x1[k], t2[k]);
           Y[k] = __dmul_rn(S.x2[k], t2[k]);
         }
-        const RareOut o = rare_pair(S.t[k], S.x1[k], S.x2[k], X[k], Y[k], EP_STAGE_U ? S.u[k] : ~0u, s_rare);
+        const RareOut o = rare_pair(S.t[k], S.x1[k], S.x2[k], X[k], Y[k], (EP_STAGE_U && !EP_IDX_TRUNC) ? S.u[k] : ~0u, s_rare);
         A.csx += o.dx;
         A.csy += o.dy;
         A.cnt += o.dcnt;
@@ -647,7 +712,7 @@ __global__ void __launch_bounds__(256) ep_pairs_debug_kernel(const __grid_consta
   __syncthreads();
   const uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
   if (i >= n) return;
-  const unsigned tab = static_cast<unsigned>(__cvta_generic_to_shared(smem_raw));
+  const unsigned tab = tab_base(smem_raw);
   const LeanConst K = make_lean_const(static_cast<unsigned>(__cvta_generic_to_shared(s_kc)));
   const uint64_t v0 = state_to_v(jump_state(P.x_begin, 2 * i, P.jump));
   unsigned vlo = unsigned(v0), vhi = unsigned(v0 >> 32);
@@ -693,7 +758,7 @@ ep_kernel(const __grid_constant__ EPParams P) {
 
   const unsigned tid = threadIdx.x;
   unsigned tab;  // opaque copy: keeps the shared base in a register (no per-use rematerialisation)
-  asm volatile("mov.u32 %0, %1;" : "=r"(tab) : "r"(static_cast<unsigned>(__cvta_generic_to_shared(smem_raw))));
+  asm volatile("mov.u32 %0, %1;" : "=r"(tab) : "r"(tab_base(smem_raw)));
   // Table -> shared memory with TMA bulk copies (cp.async.bulk, one thread,
   // completion counted on an mbarrier): one 131-KB stream at L2 bandwidth
   // instead of 16 dependent load/store rounds per thread (~8 us per launch).
@@ -920,41 +985,60 @@ ep_kernel(const __grid_constant__ EPParams P) {
     // stores), fence at system scope, signal each inbox, then wait for all
     // partials in the own inbox and fold them in rank order (deterministic,
     // identical on every rank).  No separate collective is launched.
+    //
+    // Each slot carries its call's epoch in word COMM_TAG, published with a
+    // system-scope release after the 13 data words: a rank folds only slots
+    // tagged with its own epoch, so partials of different calls never mix,
+    // and it re-reads the tags after the fold — a peer that gave up waiting
+    // (timeout) and moved on to the next call of the same parity would have
+    // changed them — so a torn read is reported (NaN + `stale`), never used.
     const CommParams& C = P.comm;
     const unsigned par = unsigned(C.epoch & 1), n = unsigned(C.nranks);
-    if (tid < 13 * n) {
-      const unsigned r = tid / 13, w = tid % 13;
+    for (unsigned i = tid; i < 13 * n; i += blockDim.x) {  // any block size covers every peer
+      const unsigned r = i / 13, w = i % 13;
       volatile double* dst = &C.inbox[r]->slot[par][C.rank][w];
       *dst = s_fin[w];
     }
     __threadfence_system();
     __syncthreads();
-    if (tid < n) {
-      unsigned long long* ctr = &C.inbox[tid]->arrived;
-      asm volatile("red.release.sys.global.add.u64 [%0], 1;" ::"l"(ctr) : "memory");
+    for (unsigned r = tid; r < n; r += blockDim.x) {
+      unsigned long long* tag = reinterpret_cast<unsigned long long*>(&C.inbox[r]->slot[par][C.rank][COMM_TAG]);
+      asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(tag), "l"(C.epoch) : "memory");
     }
+    CommInbox* own = C.inbox[C.rank];
     if (tid == 0) {
-      const unsigned long long want = C.epoch * n;
-      unsigned long long* own = &C.inbox[C.rank]->arrived;
       unsigned long long t0, now, v;
       asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
       int timed_out = 0;
-      for (;;) {
-        asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(own) : "memory");
-        if (v >= want) break;
-        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(now));
-        if (now - t0 > C.timeout_ns) { timed_out = 1; break; }
-        __nanosleep(200);
+      for (unsigned r = 0; r < n && !timed_out; ++r) {
+        const unsigned long long* tag = reinterpret_cast<const unsigned long long*>(&own->slot[par][r][COMM_TAG]);
+        for (;;) {
+          asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(tag) : "memory");
+          if (v == C.epoch) break;
+          asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(now));
+          if (now - t0 > C.timeout_ns) { timed_out = 1; break; }
+          __nanosleep(200);
+        }
       }
-      if (timed_out) atomicAdd(&C.inbox[C.rank]->timeouts, 1ull);
+      if (timed_out) atomicAdd(&own->timeouts, 1ull);
       s_last = timed_out;  // reuse: 1 = combine failed
     }
     __syncthreads();
     if (tid < 13) {
-      const volatile double* src = &C.inbox[C.rank]->slot[par][0][tid];
+      const volatile double* src = &own->slot[par][0][tid];
       double acc = 0.0;
       for (unsigned r = 0; r < n; ++r) acc += src[r * 16];  // rank order
       s_fin[tid] = acc;
+    }
+    __syncthreads();
+    if (tid == 0 && !s_last) {
+      for (unsigned r = 0; r < n; ++r) {
+        unsigned long long v;
+        const unsigned long long* tag = reinterpret_cast<const unsigned long long*>(&own->slot[par][r][COMM_TAG]);
+        asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(tag) : "memory");
+        if (v != C.epoch) s_last = 1;
+      }
+      if (s_last) atomicAdd(&own->stale, 1ull);
     }
     __syncthreads();
   }
@@ -971,13 +1055,23 @@ ep_kernel(const __grid_constant__ EPParams P) {
 }
 
 // Test hook kernel: x_{offset+i+1} via the kernel's own jump + step code.
+// The step is gen_stage's own (lcg_step_c with the unmasked carry word, or
+// lcg_step_k), so these states pin the hot loop's LCG, not a re-implementation.
+template <bool A32>
 __global__ void lcg_states_kernel(uint64_t seed, uint64_t a, uint64_t offset, uint64_t n,
                                   const __grid_constant__ JumpTable J, uint64_t* out) {
   const uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
   if (i >= n) return;
-  uint64_t v = state_to_v(jump_state(seed, offset + i, J.j));
-  v = step_v(v, a);
-  out[i] = v_to_state(v);
+  const uint64_t v = state_to_v(jump_state(seed, offset + i, J.j));
+  unsigned lo = unsigned(v), hi = unsigned(v >> 32), hd;
+  const unsigned a_lo = unsigned(a), a_hi = unsigned(a >> 32), exp_hi = 0x3FF00000u;
+#if EP_LCG_CARRY
+  lcg_step_c<A32>(lo, hi, hd, a_lo, a_hi, exp_hi);
+#else
+  lcg_step_k<A32>(lo, hi, a_lo, a_hi, exp_hi);
+  hd = hi;
+#endif
+  out[i] = v_to_state((uint64_t(hd) << 32) | lo);
 }
 
 // ------------------------------------------------------------- dispatcher
@@ -1052,6 +1146,31 @@ static void init_params(EPParams& P, uint64_t seed, uint64_t a, uint64_t pair_be
 // Lean-log table, built in 80-bit long double on the host.
 void build_log_table(std::vector<LogEntry>& tab) {
   tab.resize(LOG_TAB);
+#if EP_IDX_TRUNC
+  // truncating buckets [lo_j, lo_j + w), reference point at the centre (ep_common.cuh)
+  for (uint32_t e = 0; e < LOG_TAB; ++e) {
+    const uint32_t j = TRUNC_J0 + e;
+    if (e == 0) {                       // below the table -> moderate X, Y -> exact rare path
+      tab[e].T = 60.0;
+      tab[e].inv = 0.0;
+    } else if (j < LOG_IDX_MAX - 1) {   // real bucket of t' in [2^-18, 1/4 - w)
+      const int E = int(j >> LOG_K) - 1023;
+      const long double centre =
+          ldexpl(1.0L + ((long double)(j & ((1u << LOG_K) - 1)) + 0.5L) / (1 << LOG_K), E);
+      const float inv = (float)(1.0L / centre);
+      tab[e].inv = (double)inv;
+      tab[e].T = (double)(2.0L * logl((long double)inv * 0.25L));  // -2 ln(4 t') at r = 0
+    } else if (j <= LOG_IDX_MAX) {      // [1/4 - w, 1/4 + w), reference point 1/4 itself (T = 0,
+                                        // r = 4t' - 1 exact): L = -2 ln(1 + r) has no cancellation
+                                        // as t' -> 1/4; t' = 1/4 -> L = 0; above -> L < 0 -> NaN
+      tab[e].T = 0.0;
+      tab[e].inv = 4.0;
+    } else {                            // reject sentinels up to t' = 1/2
+      tab[e].T = 0x1p1000;
+      tab[e].inv = 0.0;
+    }
+  }
+#else
   for (uint32_t u = 0; u < LOG_N; ++u) {
     const uint32_t idx = LOG_IDX_MIN + u;
     const int E = int(idx >> LOG_K) - 1023;
@@ -1066,6 +1185,7 @@ void build_log_table(std::vector<LogEntry>& tab) {
   }
   tab[LOG_TINY].T = 60.0;  // t' below the table -> moderate X, Y -> exact rare path
   tab[LOG_TINY].inv = 0.0;
+#endif
 }
 
 namespace {
@@ -1129,26 +1249,24 @@ int device_state(int device, const LogEntry** table, int* sms) {
   return 0;
 }
 
+// One workspace per (device, stream), sized once for the largest grid any
+// configuration can launch (sms x 32 blocks) and never reallocated, so a
+// pointer handed to one host thread can never be freed under another's
+// pending launch.
 static int workspace(int device, cudaStream_t stream, int blocks, EPPartial** partials, unsigned** counter) {
   std::lock_guard<std::mutex> lk(g_mu);
   for (auto& w : g_ws) {
     if (w.device == device && w.stream == stream) {
-      if (w.capacity < blocks) {
-        cudaError_t e = cudaStreamSynchronize(stream);
-        if (e != cudaSuccess) return set_cuda_error(e, "cudaStreamSynchronize");
-        cudaFree(w.partials);
-        w.partials = nullptr;
-        e = cudaMalloc(&w.partials, sizeof(EPPartial) * blocks);
-        if (e != cudaSuccess) return set_cuda_error(e, "cudaMalloc(partials)");
-        w.capacity = blocks;
-      }
+      if (w.capacity < blocks) return set_error(HPL_EINVAL, "grid of %d blocks exceeds the workspace (%d)", blocks, w.capacity);
       *partials = w.partials;
       *counter = w.counter;
       return 0;
     }
   }
-  Workspace w{device, stream, nullptr, nullptr, blocks};
-  cudaError_t e = cudaMalloc(&w.partials, sizeof(EPPartial) * blocks);
+  const int cap = g_dev[device].sms * EP_MAX_BLOCKS_PER_SM;
+  if (blocks > cap) return set_error(HPL_EINVAL, "grid of %d blocks exceeds the workspace (%d)", blocks, cap);
+  Workspace w{device, stream, nullptr, nullptr, cap};
+  cudaError_t e = cudaMalloc(&w.partials, sizeof(EPPartial) * cap);
   if (e != cudaSuccess) return set_cuda_error(e, "cudaMalloc(partials)");
   e = cudaMalloc(&w.counter, sizeof(unsigned));
   if (e == cudaSuccess) e = cudaMemset(w.counter, 0, sizeof(unsigned));
@@ -1237,6 +1355,32 @@ int launch_ep(int device, uint64_t seed, uint64_t a, uint64_t pair_begin, uint64
   return 0;
 }
 
+// hpl_shutdown(): free the log tables and EP workspaces of every device
+// (each device synchronised first); they are re-created on the next call.
+int release_ep_state() {
+  std::lock_guard<std::mutex> lk(g_mu);
+  int prev = -1;
+  cudaGetDevice(&prev);
+  cudaError_t first = cudaSuccess;
+  for (auto& w : g_ws) {
+    cudaSetDevice(w.device);
+    cudaError_t e = cudaStreamSynchronize(w.stream);
+    if (e != cudaSuccess && first == cudaSuccess) first = e;
+    cudaFree(w.partials);
+    cudaFree(w.counter);
+  }
+  g_ws.clear();
+  for (size_t d = 0; d < g_dev.size(); ++d)
+    if (g_dev[d].table) {
+      cudaSetDevice(int(d));
+      cudaDeviceSynchronize();
+      cudaFree(g_dev[d].table);
+      g_dev[d].table = nullptr;
+    }
+  if (prev >= 0) cudaSetDevice(prev);
+  return first == cudaSuccess ? 0 : set_cuda_error(first, "hpl_shutdown: synchronize");
+}
+
 unsigned long long launch_count() {
   std::lock_guard<std::mutex> lk(g_mu);
   return g_launches;
@@ -1271,7 +1415,10 @@ int launch_lcg_states(uint64_t seed, uint64_t a, uint64_t offset, uint64_t n, ui
   const int thr = 256;
   const uint64_t blocks = (n + thr - 1) / thr;
   if (blocks == 0) return 0;
-  lcg_states_kernel<<<unsigned(blocks), thr, 0, stream>>>(seed & MASK46, a, offset, n, J, dev_out);
+  if ((a >> 32) == 0)
+    lcg_states_kernel<true><<<unsigned(blocks), thr, 0, stream>>>(seed & MASK46, a, offset, n, J, dev_out);
+  else
+    lcg_states_kernel<false><<<unsigned(blocks), thr, 0, stream>>>(seed & MASK46, a, offset, n, J, dev_out);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return set_cuda_error(e, "lcg_states_kernel launch");
   return 0;

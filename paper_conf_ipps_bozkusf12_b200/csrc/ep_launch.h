@@ -42,6 +42,7 @@ int launch_ep(int device, uint64_t seed, uint64_t a, uint64_t pair_begin, uint64
 int launch_lcg_states(uint64_t seed, uint64_t a, uint64_t offset, uint64_t n, uint64_t* dev_out,
                       cudaStream_t stream);
 unsigned long long launch_count();
+int release_ep_state();
 int launch_pairs_debug(int device, uint64_t seed, uint64_t a, uint64_t pair_begin, uint64_t n,
                        double* dev_out, cudaStream_t stream);
 

@@ -7,6 +7,7 @@
 
 #include <cstdarg>
 #include <cstdio>
+#include <cstddef>
 #include <cstring>
 #include <deque>
 #include <mutex>
@@ -73,6 +74,50 @@ static int shard_range(int M, int rank, int nranks, uint64_t* begin, uint64_t* n
 
 using namespace hplep;
 
+// ---- device allocator (SURVEY §8(b) "memory ownership"): cudaMalloc unless a
+// caller installs one, e.g. the Python binding installs torch's caching
+// allocator (torch.cuda.caching_allocator_alloc/delete), so arrays draw from
+// the same pool as the caller's tensors without a synchronous cudaMalloc.
+namespace {
+std::mutex g_alloc_mu;
+hpl_alloc_fn g_alloc = nullptr;
+hpl_free_fn g_free = nullptr;
+void* g_alloc_ctx = nullptr;
+
+struct DevAlloc {
+  hpl_free_fn free = nullptr;  // nullptr: cudaFree
+  void* ctx = nullptr;
+};
+
+int dev_alloc(void** p, size_t bytes, int device, DevAlloc* how) {
+  hpl_alloc_fn a;
+  {
+    std::lock_guard<std::mutex> lk(g_alloc_mu);
+    a = g_alloc;
+    how->free = g_free;
+    how->ctx = g_alloc_ctx;
+  }
+  if (a) {
+    *p = a(bytes, device, how->ctx);
+    if (!*p) return set_error(HPL_ENOMEM, "device allocator returned NULL for %zu bytes", bytes);
+    return 0;
+  }
+  how->free = nullptr;
+  cudaError_t e = cudaMalloc(p, bytes);
+  if (e != cudaSuccess) return set_cuda_error(e, "cudaMalloc");
+  return 0;
+}
+
+cudaError_t dev_free(void* p, size_t bytes, int device, const DevAlloc& how) {
+  if (!p) return cudaSuccess;
+  if (how.free) {
+    how.free(p, bytes, device, how.ctx);
+    return cudaSuccess;
+  }
+  return cudaFree(p);
+}
+}  // namespace
+
 struct hpl_array_s {
   hpl_dtype t;
   int ndim;
@@ -85,6 +130,7 @@ struct hpl_array_s {
   int device;
   cudaStream_t stream;
   int valid;
+  DevAlloc how;  // how the device copy was allocated (freed the same way)
 };
 
 static size_t dtype_size(int t) {
@@ -187,15 +233,16 @@ int hpl_array_alloc(hpl_array* out, hpl_dtype t, int ndim, const int64_t* dims, 
   a->nbytes = size_t(count) * es;
   a->device = device;
   a->stream = nullptr;
-  cudaError_t e = cudaMalloc(&a->dev, a->nbytes);
-  if (e != cudaSuccess) { delete a; return set_cuda_error(e, "cudaMalloc(array)"); }
+  int arc = dev_alloc(&a->dev, a->nbytes, device, &a->how);
+  if (arc) { delete a; return arc; }
+  cudaError_t e;
   if (host_ptr) {
     a->host = host_ptr;
     a->host_owned = false;
     a->valid = HPL_HOST;
   } else {
     e = cudaMallocHost(&a->host, a->nbytes);
-    if (e != cudaSuccess) { cudaFree(a->dev); delete a; return set_cuda_error(e, "cudaMallocHost(array)"); }
+    if (e != cudaSuccess) { dev_free(a->dev, a->nbytes, device, a->how); delete a; return set_cuda_error(e, "cudaMallocHost(array)"); }
     a->host_owned = true;
     a->valid = HPL_HOST | HPL_DEVICE;
   }
@@ -207,7 +254,7 @@ int hpl_array_free(hpl_array a) {
   if (!a) return HPL_OK;
   DeviceGuard g(a->device);
   cudaError_t e1 = a->stream ? cudaStreamSynchronize(a->stream) : cudaDeviceSynchronize();
-  cudaError_t e2 = cudaFree(a->dev);
+  cudaError_t e2 = dev_free(a->dev, a->nbytes, a->device, a->how);
   cudaError_t e3 = a->host_owned ? cudaFreeHost(a->host) : cudaSuccess;
   delete a;
   if (e1 != cudaSuccess) return set_cuda_error(e1, "hpl_array_free: synchronize");
@@ -301,7 +348,8 @@ struct hpl_comm_s {
 
 int hpl_comm_create(hpl_comm* out, int rank, int nranks, int device, void* handle_out) {
   if (!out || !handle_out) return set_error(HPL_EINVAL, "NULL argument");
-  if (nranks < 1 || nranks > hplep::COMM_MAX_RANKS) return set_error(HPL_EINVAL, "nranks must be in [1, %d]", hplep::COMM_MAX_RANKS);
+  if (nranks < 1 || nranks > hplep::COMM_MAX_RANKS || (nranks & (nranks - 1)))
+    return set_error(HPL_EINVAL, "nranks must be a power of two in [1, %d] (equal EP shards)", hplep::COMM_MAX_RANKS);
   if (rank < 0 || rank >= nranks) return set_error(HPL_EINVAL, "rank out of range");
   if (device < 0) {
     int rc = current_device(&device);
@@ -397,12 +445,14 @@ int hpl_comm_status(hpl_comm c, void* stream, uint64_t* epoch, uint64_t* timeout
   DeviceGuard g(c->device);
   if (g.rc) return g.rc;
   cudaError_t e = cudaStreamSynchronize(static_cast<cudaStream_t>(stream));
-  unsigned long long t = 0;
-  if (e == cudaSuccess) e = cudaMemcpy(&t, &c->own->timeouts, sizeof(t), cudaMemcpyDeviceToHost);
+  unsigned long long w[2] = {0, 0};  // {stale, timeouts}
+  static_assert(offsetof(hplep::CommInbox, timeouts) == offsetof(hplep::CommInbox, stale) + 8, "layout");
+  if (e == cudaSuccess) e = cudaMemcpy(w, &c->own->stale, sizeof(w), cudaMemcpyDeviceToHost);
   if (e != cudaSuccess) return set_cuda_error(e, "comm status");
   *epoch = c->epoch;
-  *timeouts = t;
-  if (t) return set_error(HPL_ECUDA, "fused combine: %llu call(s) timed out waiting for a peer", t);
+  *timeouts = w[0] + w[1];
+  if (w[1]) return set_error(HPL_ECUDA, "fused combine: %llu call(s) timed out waiting for a peer", w[1]);
+  if (w[0]) return set_error(HPL_ECUDA, "fused combine: %llu call(s) saw a peer's slot change during the fold", w[0]);
   return HPL_OK;
 }
 
@@ -422,6 +472,21 @@ int hpl_ep_eval(int M, uint64_t seed, uint64_t a, int rank, int nranks, hpl_arra
   return HPL_OK;
 }
 
+}  // extern "C"
+namespace {
+struct RunCache {
+  static constexpr int N = 64;
+  hpl_array a[N] = {nullptr};
+  void release() {
+    for (auto& x : a)
+      if (x) { hpl_array_free(x); x = nullptr; }
+  }
+  ~RunCache() { release(); }
+};
+thread_local RunCache t_run;
+}  // namespace
+extern "C" {
+
 int hpl_ep_run(int M, uint64_t seed, uint64_t a, double* sx, double* sy, uint64_t q[10]) {
   if (!sx || !sy || !q) return set_error(HPL_EINVAL, "NULL output pointer");
   uint64_t b0, n0;
@@ -432,15 +497,16 @@ int hpl_ep_run(int M, uint64_t seed, uint64_t a, double* sx, double* sy, uint64_
   rc = current_device(&dev);
   if (rc) return rc;
   // one cached 13-word Array per thread and device (the paper's Array with
-  // a library-owned host copy)
-  thread_local hpl_array cache[64] = {nullptr};
-  if (dev >= 64) return set_error(HPL_EINVAL, "device index too large");
-  if (!cache[dev]) {
+  // a library-owned host copy); freed at thread exit or by
+  // hpl_shutdown()
+  if (dev >= RunCache::N) return set_error(HPL_EINVAL, "device index too large");
+  hpl_array& slot = t_run.a[dev];
+  if (!slot) {
     int64_t d = 13;
-    rc = hpl_array_alloc(&cache[dev], HPL_F64, 1, &d, nullptr, dev);
+    rc = hpl_array_alloc(&slot, HPL_F64, 1, &d, nullptr, dev);
     if (rc) return rc;
   }
-  hpl_array out = cache[dev];
+  hpl_array out = slot;
   rc = hpl_ep_eval(M, seed, a, 0, 1, out);
   if (rc) return rc;
   rc = hpl_array_sync(out, HPL_HOST, HPL_READ);  // 104-byte D2H, blocking
@@ -459,15 +525,20 @@ int hpl_lcg_states(uint64_t seed, uint64_t a, uint64_t offset, uint64_t n, uint6
   if (n > (uint64_t(1) << 28)) return set_error(HPL_EINVAL, "n must be <= 2^28");
   if (n == 0) return HPL_OK;
   if (!host_out) return set_error(HPL_EINVAL, "host_out is NULL");
-  uint64_t* d = nullptr;
-  cudaError_t e = cudaMalloc(&d, n * sizeof(uint64_t));
-  if (e != cudaSuccess) return set_cuda_error(e, "cudaMalloc(states)");
-  rc = launch_lcg_states(seed, a, offset, n, d, nullptr);
+  int dev;
+  rc = current_device(&dev);
+  if (rc) return rc;
+  void* d = nullptr;
+  DevAlloc how;
+  rc = dev_alloc(&d, n * sizeof(uint64_t), dev, &how);
+  if (rc) return rc;
+  rc = launch_lcg_states(seed, a, offset, n, static_cast<uint64_t*>(d), nullptr);
   if (!rc) {
-    e = cudaMemcpy(host_out, d, n * sizeof(uint64_t), cudaMemcpyDeviceToHost);
+    cudaError_t e = cudaMemcpy(host_out, d, n * sizeof(uint64_t), cudaMemcpyDeviceToHost);
     if (e != cudaSuccess) rc = set_cuda_error(e, "cudaMemcpy(states)");
   }
-  cudaFree(d);
+  cudaDeviceSynchronize();
+  dev_free(d, n * sizeof(uint64_t), dev, how);
   return rc;
 }
 
@@ -653,8 +724,25 @@ int hpl_eval(const char* name, int ndim, const int64_t* global, const int64_t* l
   if (rc) return rc;
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return set_cuda_error(e, name);
-  for (int i = 0; i < nargs; ++i)
-    if (sig[i].array && (sig[i].mode & HPL_WRITE)) args[i].array->valid = HPL_DEVICE;
+  // a written array whose own stream differs from the launch stream: order its
+  // stream after the kernel, so a later hpl_array_sync(HOST) on that stream
+  // (or any work the caller queues there) sees the kernel's output
+  cudaEvent_t done = nullptr;
+  for (int i = 0; i < nargs; ++i) {
+    if (!sig[i].array || !(sig[i].mode & HPL_WRITE)) continue;
+    hpl_array a = args[i].array;
+    if (a->stream != stream) {
+      if (!done) {
+        e = cudaEventCreateWithFlags(&done, cudaEventDisableTiming);
+        if (e == cudaSuccess) e = cudaEventRecord(done, stream);
+        if (e != cudaSuccess) return set_cuda_error(e, "hpl_eval: completion event");
+      }
+      e = cudaStreamWaitEvent(a->stream, done, 0);
+      if (e != cudaSuccess) { cudaEventDestroy(done); return set_cuda_error(e, "cudaStreamWaitEvent"); }
+    }
+    a->valid = HPL_DEVICE;
+  }
+  if (done) cudaEventDestroy(done);  // released once the recorded work completes
   return HPL_OK;
 }
 
@@ -737,15 +825,46 @@ int hpl_ep_pairs_debug(uint64_t seed, uint64_t a, uint64_t pair_begin, uint64_t 
   int dev;
   rc = current_device(&dev);
   if (rc) return rc;
-  double* d = nullptr;
-  cudaError_t e = cudaMalloc(&d, n * 4 * sizeof(double));
-  if (e != cudaSuccess) return set_cuda_error(e, "cudaMalloc(debug)");
-  rc = launch_pairs_debug(dev, seed, a, pair_begin, n, d, nullptr);
+  void* d = nullptr;
+  DevAlloc how;
+  rc = dev_alloc(&d, n * 4 * sizeof(double), dev, &how);
+  if (rc) return rc;
+  rc = launch_pairs_debug(dev, seed, a, pair_begin, n, static_cast<double*>(d), nullptr);
   if (!rc) {
-    e = cudaMemcpy(host_out, d, n * 4 * sizeof(double), cudaMemcpyDeviceToHost);
+    cudaError_t e = cudaMemcpy(host_out, d, n * 4 * sizeof(double), cudaMemcpyDeviceToHost);
     if (e != cudaSuccess) rc = set_cuda_error(e, "cudaMemcpy(debug)");
   }
-  cudaFree(d);
+  cudaDeviceSynchronize();
+  dev_free(d, n * 4 * sizeof(double), dev, how);
+  return rc;
+}
+
+int hpl_set_device_allocator(hpl_alloc_fn alloc, hpl_free_fn free_fn, void* ctx) {
+  if ((alloc == nullptr) != (free_fn == nullptr)) return set_error(HPL_EINVAL, "alloc and free must both be set or both be NULL");
+  std::lock_guard<std::mutex> lk(g_alloc_mu);
+  g_alloc = alloc;
+  g_free = free_fn;
+  g_alloc_ctx = alloc ? ctx : nullptr;
+  return HPL_OK;
+}
+
+int hpl_shutdown(void) {
+  t_run.release();
+  int rc = release_ep_state();
+  {
+    std::lock_guard<std::mutex> lk(g_red_mu);
+    for (auto& w : g_red) {
+      DeviceGuard g(w.device);
+      cudaStreamSynchronize(w.stream);
+      cudaFree(w.ws.partials);
+      cudaFree(w.ws.counter);
+    }
+    g_red.clear();
+  }
+  std::lock_guard<std::mutex> lk(g_alloc_mu);
+  g_alloc = nullptr;
+  g_free = nullptr;
+  g_alloc_ctx = nullptr;
   return rc;
 }
 

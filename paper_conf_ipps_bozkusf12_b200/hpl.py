@@ -11,8 +11,10 @@ on a non-zero status; the C status code is ``err.code``.
 """
 from __future__ import annotations
 
+import atexit
 import ctypes
 import os
+import sys
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
 # HPL_LIB: development override to load an A/B build variant of the library
@@ -37,9 +39,16 @@ EXPORTS = (
     "hpl_ep_pairs_debug",
     "hpl_comm_create", "hpl_comm_open", "hpl_comm_set_timeout", "hpl_comm_free",
     "hpl_ep_run_fused", "hpl_comm_status",
+    "hpl_set_device_allocator", "hpl_shutdown",
 )
 HPL_COMM_HANDLE_BYTES, HPL_COMM_MAX_RANKS = 64, 8
 HPL_ARG_ARRAY, HPL_ARG_F64, HPL_ARG_F32, HPL_ARG_I64, HPL_ARG_I32 = 0, 1, 2, 3, 4
+
+
+# hpl_alloc_fn / hpl_free_fn (include/hpl.h)
+_ALLOC_T = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_int, ctypes.c_void_p)
+_FREE_T = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_size_t, ctypes.c_int, ctypes.c_void_p)
+_allocator = None  # the installed callbacks (kept alive here)
 
 
 class HplArg(ctypes.Structure):
@@ -103,12 +112,16 @@ def _load() -> ctypes.CDLL:
         "hpl_comm_free": (c_int, [c_void_p]),
         "hpl_ep_run_fused": (c_int, [c_void_p, c_int, c_u64, c_u64, c_void_p, c_void_p]),
         "hpl_comm_status": (c_int, [c_void_p, c_void_p, P(c_u64), P(c_u64)]),
+        "hpl_set_device_allocator": (c_int, [_ALLOC_T, _FREE_T, c_void_p]),
+        "hpl_shutdown": (c_int, []),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)
         f.restype = res
         f.argtypes = args
     _lib = lib
+    if "torch" in sys.modules:  # the caller uses torch: arrays share its caching allocator
+        use_torch_allocator()
     return lib
 
 
@@ -123,6 +136,50 @@ def _check(rc: int, func: str) -> None:
 
 def lib() -> ctypes.CDLL:
     return _load()
+
+
+# ------------------------------------------------- device memory / state
+def hpl_set_device_allocator(alloc=None, free=None) -> None:
+    """Install Python callables alloc(nbytes, device) -> int pointer and
+    free(ptr, nbytes, device) as the library's device allocator (both None:
+    back to cudaMalloc)."""
+    global _allocator
+    lib = _load()
+    if alloc is None and free is None:
+        _check(lib.hpl_set_device_allocator(_ALLOC_T(), _FREE_T(), None), "hpl_set_device_allocator")
+        _allocator = None
+        return
+    cb = (_ALLOC_T(lambda n, dev, ctx: alloc(n, dev) or None),
+          _FREE_T(lambda p, n, dev, ctx: free(p, n, dev)))
+    _check(lib.hpl_set_device_allocator(cb[0], cb[1], None), "hpl_set_device_allocator")
+    _allocator = cb
+
+
+def use_torch_allocator() -> None:
+    """Route hpl_array device memory through torch's CUDA caching allocator
+    (SURVEY §8(b) memory ownership; reading B1).  Installed
+    automatically when torch is imported before the library is loaded."""
+    import torch
+
+    def alloc(n, dev):
+        return torch.cuda.caching_allocator_alloc(n, device=dev)
+
+    def free(p, n, dev):
+        torch.cuda.caching_allocator_delete(p)
+
+    hpl_set_device_allocator(alloc, free)
+
+
+def hpl_shutdown() -> None:
+    """Free every library-owned buffer (see include/hpl.h); registered at exit
+    so torch-allocated arrays are returned while the interpreter is alive."""
+    global _allocator
+    if _lib is not None:
+        _check(_lib.hpl_shutdown(), "hpl_shutdown")
+        _allocator = None
+
+
+atexit.register(lambda: _lib is not None and _lib.hpl_shutdown())
 
 
 # ------------------------------------------------------------------ devices

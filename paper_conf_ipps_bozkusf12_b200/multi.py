@@ -113,8 +113,13 @@ class FusedComm:
         return hpl.hpl_comm_status(self.comm, torch.cuda.current_stream(self.device).cuda_stream)
 
     def close(self) -> None:
+        """Collective: every rank drains its own kernels, then a barrier makes
+        sure no peer kernel can still be storing into (or reading) any inbox,
+        then the mappings and the own inbox are released."""
         if self.comm:
             torch.cuda.synchronize(self.device)
+            if self.world > 1 and dist.is_initialized():
+                dist.barrier(group=self.group)
             hpl.hpl_comm_free(self.comm)
             self.comm = None
 

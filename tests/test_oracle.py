@@ -8,6 +8,8 @@ a wrong batch seed or a wrong bin truncation each fails at least one test
 (DESIGN.md §3 maps mistakes to pins).
 """
 import math
+
+import numpy as np
 import random
 from decimal import Decimal, localcontext
 
@@ -261,3 +263,123 @@ def test_worked_example_first_pairs():
             X, Y = float(Decimal(x1) * f), float(Decimal(x2) * f)
             assert abs(X - float(r[1])) <= 4 * math.ulp(X) and abs(Y - float(r[2])) <= 4 * math.ulp(Y)
             assert int(max(abs(X), abs(Y))) == int(r[3])
+
+
+# ------------------------------------ C10 / C7 additions: compensated sums, margin
+def test_csum_adversarial_sequences(oracle_mod):
+    """Reading R10 (C10): the oracle's Neumaier sum is the exactly rounded sum
+    (math.fsum) on cancellation patterns where plain, and Kahan, summation fail."""
+    cases = [
+        [1e16, 1.0, -1e16],                       # plain: 0
+        [1.0, 1e100, 1.0, -1e100],                # Kahan: 0, Neumaier: 2
+        [2.0 ** 53, 1.0, 1.0, 1.0, -(2.0 ** 53)],  # plain: 2 (ties to even), exact 3
+        [0.1] * 10 + [-1.0],                      # classic 1-ulp residue
+    ]
+    for seq in cases:
+        assert oracle_mod.csum(seq) == math.fsum(seq), seq
+    assert oracle_mod.csum([]) == 0.0
+
+
+def test_csum_long_random_sequence(oracle_mod):
+    """2^20 N(0,1)-like terms plus large cancelling pairs: within 1 ulp of
+    fsum, while plain sequential summation is off by far more (the pin
+    discriminates a `s += v` mutation)."""
+    rng = random.Random(2024)
+    seq = []
+    for i in range(1 << 20):
+        seq.append(rng.gauss(0.0, 1.0))
+        if i % 4096 == 0:
+            big = rng.uniform(1e6, 1e9)
+            seq += [big, -big * (1 + 2.0 ** -40)]
+    exact = math.fsum(seq)
+    plain = 0.0
+    for v in seq:
+        plain += v
+    assert abs(oracle_mod.csum(seq) - exact) <= math.ulp(exact)
+    assert abs(plain - exact) > 10 * math.ulp(exact)
+
+
+def test_oracle_deviates_vs_decimal(oracle_mod):
+    """The exported per-pair deviates (the same gauss_pair the runs use) are
+    within 2 ulp of 50-digit decimal X, Y and their bins match, pair by pair."""
+    M = 11
+    X, Y, l = oracle_mod.pairs(NPB_SEED, NPB_A, 0, 1 << M)
+    x = NPB_SEED
+    with localcontext() as ctx:
+        ctx.prec = 50
+        for i in range(1 << M):
+            x = NPB_A * x % MOD46
+            x1 = 2.0 * (x * 2.0 ** -46) - 1.0
+            x = NPB_A * x % MOD46
+            x2 = 2.0 * (x * 2.0 ** -46) - 1.0
+            t = x1 * x1 + x2 * x2
+            if t > 1.0:
+                assert l[i] == -1
+                continue
+            f = (Decimal(-2) * Decimal(t).ln() / Decimal(t)).sqrt()
+            Xd, Yd = float(Decimal(x1) * f), float(Decimal(x2) * f)
+            assert abs(X[i] - Xd) <= 2 * math.ulp(Xd) and abs(Y[i] - Yd) <= 2 * math.ulp(Yd)
+            assert l[i] == int(max(abs(X[i]), abs(Y[i])))
+
+
+@pytest.mark.parametrize("M,mk", [(20, 20), (20, 12)])
+def test_run_sums_are_compensated(oracle_mod, M, mk):
+    """R10 at run level: the oracle's sx, sy equal the exactly rounded sum of its
+    own deviates to <= 2 ulp (one batch, and 256 batches combined in order),
+    whereas plain sequential summation of the same deviates is off by > 10 ulp."""
+    X, Y, l = oracle_mod.pairs(NPB_SEED, NPB_A, 0, 1 << M)
+    r = oracle_mod.run(M, NPB_SEED, NPB_A, mk=mk, threads=4, margin=False)
+    assert r.gc == int((l >= 0).sum())
+    for got, v in ((r.sx, X), (r.sy, Y)):
+        exact = math.fsum(v.tolist())
+        assert abs(got - exact) <= 2 * math.ulp(exact), (got, exact)
+    plain = 0.0
+    for v in X.tolist():
+        plain += v
+    exact = math.fsum(X.tolist())
+    assert abs(plain - exact) > 10 * math.ulp(exact)
+
+
+def _margin_py(X, Y, l):
+    """Reading R7 recomputed here: min over accepted pairs of |m - n| / ulp(m),
+    n = nearest integer of m = max(|X|,|Y|), counted when 1 <= n <= 10."""
+    best = 1e300
+    for xv, yv, lv in zip(X.tolist(), Y.tolist(), l.tolist()):
+        if lv < 0:
+            continue
+        m = max(abs(xv), abs(yv))
+        n = round(m)
+        if 1 <= n <= 10:
+            best = min(best, abs(m - n) / math.ulp(m))
+    return best
+
+
+@pytest.mark.parametrize("seed,begin,n", [(NPB_SEED, 0, 1 << 15), (NPB_SEED, 2 ** 30 + 77, 1 << 15),
+                                          (1, 0, 1 << 14), ((1 << 46) - 1, 4321, 1 << 14)])
+def test_bin_margin_matches_recomputation(oracle_mod, seed, begin, n):
+    """C7: the oracle's min_margin_ulp equals the margin recomputed in Python
+    from its deviates (catches a tracker that is never updated or mis-measured)."""
+    X, Y, l = oracle_mod.pairs(seed, NPB_A, begin, n)
+    r = oracle_mod.run_pairs(seed, NPB_A, begin, n, margin=True)
+    assert r.min_margin_ulp == _margin_py(X, Y, l)
+    assert r.min_margin_ulp < 1e300
+
+
+def test_bin_margin_locates_the_closest_pair(oracle_mod):
+    """C7 on a constructed small-margin window: find the pair of 2^18 closest to a
+    bin boundary, then a 64-pair window around it reports exactly that margin
+    and a window without it reports a larger one."""
+    n = 1 << 18
+    X, Y, l = oracle_mod.pairs(NPB_SEED, NPB_A, 0, n)
+    m = np.maximum(np.abs(X), np.abs(Y))
+    near = np.rint(m)
+    ok = (l >= 0) & (near >= 1) & (near <= 10)
+    d = np.where(ok, np.abs(m - near) / np.spacing(m), np.inf)
+    i = int(np.argmin(d))
+    assert d[i] < 2.0 ** 40   # a genuinely small margin at this size (~2^-12 relative)
+    lo = max(0, i - 32)
+    w = oracle_mod.run_pairs(NPB_SEED, NPB_A, lo, 64, margin=True)
+    assert w.min_margin_ulp == float(d[i])
+    far = oracle_mod.run_pairs(NPB_SEED, NPB_A, i + 1, 64, margin=True)
+    assert far.min_margin_ulp > float(d[i])
+    assert oracle_mod.bin_margin(float(m[i])) == float(d[i])

@@ -55,6 +55,7 @@ FP64 = ("DFMA", "DMUL", "DADD", "DSETP", "DMNMX")
 mix = collections.Counter()
 reads = collections.Counter()
 prev_reuse = {}
+bank_cyc = 0.0  # RF-bank issue model: max(distinct even, distinct odd) registers read, >= 1
 for a, i in hot:
     s = re.sub(r"^@!?U?P\w+\s+", "", i)
     op = s.split()[0]
@@ -66,6 +67,7 @@ for a, i in hot:
         nd = 0
     srcs = args[nd:]
     new_reuse = {}
+    regs = set()
     for slot, x in enumerate(srcs):
         m = re.match(r"^\[?-?\|?-?(R\d+)\|?(\.reuse)?", x)
         if not m or m.group(1) == "RZ":
@@ -76,14 +78,20 @@ for a, i in hot:
         if prev_reuse.get(slot) == m.group(1):
             w = 0
         reads[base] += w
+        if w:
+            r0 = int(m.group(1)[1:])
+            regs.update(range(r0, r0 + w))
         if m.group(2):
             new_reuse[slot] = m.group(1)
     prev_reuse = new_reuse
+    ev = sum(1 for r in regs if r % 2 == 0)
+    bank_cyc += max(1, ev, len(regs) - ev)
 n = len(hot)
 print(f"loop 0x{lo:x}-0x{hi:x}: {n} hot instructions = {n / ppi:.2f}/pair "
       f"({len(cold)} cold dropped); reads {sum(reads.values()) / ppi:.1f}/pair")
 fp = sum(v for k, v in mix.items() if k.split(".")[0] in FP64)
 print(f"  FP64 {fp / ppi:.2f}/pair, other {(n - fp) / ppi:.2f}/pair")
+print(f"  RF-bank issue model: {bank_cyc / ppi:.1f} cycles/warp-pair (FP64 pipe floor {2 * fp / ppi:.1f})")
 for k, v in mix.most_common():
     print(f"  {k:24s} {v / ppi:5.2f}")
 print("  reads by opcode:")
