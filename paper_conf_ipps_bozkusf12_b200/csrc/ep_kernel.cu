@@ -59,7 +59,12 @@ __device__ __forceinline__ double rsqrt_approx(double p) {
 // Shared-memory address of the log-table entry of t' (high word H).  `tabb` is
 // the table base, pre-biased by -TRUNC_J0 entries in the truncating mode.
 __device__ __forceinline__ unsigned tab_addr(unsigned H, unsigned tabb) {
-#if EP_IDX_TRUNC
+#if EP_IDX_TRUNC && EP_T_FMA == 2
+  // H + 1: the fused t' with high word 0x3FCFFFFF (just below 1/4) shares the
+  // NaN bucket of [1/4, 1/4 + w) -> rare path (exact acceptance); other t'
+  // move at most one high-word step (|r| <= 2^-10 + 2^-20)
+  return ((max(H + 1u, TRUNC_HLO) >> LOG_SHIFT) << 4) + tabb;
+#elif EP_IDX_TRUNC
   return ((max(H, TRUNC_HLO) >> LOG_SHIFT) << 4) + tabb;
 #else
   return (min((H + LOG_ADD) >> LOG_SHIFT, LOG_N) << 4) + tabb;
@@ -219,13 +224,21 @@ struct RareOut {
 // u = ~0u the index is recomputed here (the stage then need not keep it live).
 __device__ __noinline__ RareOut rare_pair(double t, double x1, double x2, double X, double Y,
                                           unsigned u, unsigned long long* s_rare) {
-  if (t > 0.25) return RareOut{0.0, 0.0, 0u};  // rejected (never routed here by the fast path)
+#if EP_T_FMA
+  // the caller's t' is fused: recompute NPB's t' = RN(RN(x1'^2) + RN(x2'^2));
+  // where the two differ, X, Y are recomputed from NPB's t' below
+  const double tf = t;
+  t = __dadd_rn(__dmul_rn(x1, x1), __dmul_rn(x2, x2));
+#else
+  const double tf = t;
+#endif
+  if (t > 0.25) return RareOut{0.0, 0.0, 0u};  // rejected
 #if EP_IDX_TRUNC
   (void)u;
-  if (below_table(t)) {
+  if (below_table(t) || t != tf || X != X) {  // (NaN: EP_T_FMA == 2's bucket at 1/4)
 #else
   if (u == ~0u) u = (static_cast<unsigned>(__double2hiint(t)) + LOG_ADD) >> LOG_SHIFT;  // wraps below the table
-  if (u >= LOG_N) {
+  if (u >= LOG_N || t != tf) {
 #endif  // t below the table: NPB's formula, libdevice log/sqrt, on
     // the unscaled t = 4 t', x = 2 x' (exact)
     const double tt = 4.0 * t;
@@ -454,6 +467,16 @@ constexpr int kLoopUnroll = EP_LOOP_UNROLL;  // (#pragma arguments are not macro
 #ifndef EP_RARE_VOTE
 #define EP_RARE_VOTE 1 // 1: rare-path branch on a warp vote (needs warp-uniform trip counts)
 #endif
+#ifndef EP_LOG_DEG4
+#define EP_LOG_DEG4 1  // 1: degree-4 series for -2 ln(1+r) (K >= 9: |error| <= (2/5) 2^-50 absolute in L)
+#endif
+#ifndef EP_T_FMA
+#define EP_T_FMA 0     // 1: t' = fma(x1', x1', RN(x2'^2)) (<= 1 ulp from NPB's t'); t' within 2^-20 of 1/4
+#endif                 //    goes to the rare path, which recomputes NPB's t' and decides acceptance exactly
+#ifndef EP_JUMP_WIN
+#define EP_JUMP_WIN 1  // 1: per-thread skip-ahead by 4-bit windows (shared-memory table)
+#endif
+constexpr int EP_WIN_N = (NJUMP + 3) / 4;  // 12 windows cover 2 p0 < 2^46
 #ifndef EP_PIPE
 #define EP_PIPE 1      // 1: software-pipeline generation of group g+1 under the transform of group g
 #endif
@@ -504,6 +527,8 @@ __device__ __forceinline__ void gen_stage(unsigned& vlo, unsigned& vhi, const EP
     const double s1 = __dmul_rn(S.x1[k], S.x1[k]), s2 = __dmul_rn(S.x2[k], S.x2[k]);
     S.t[k] = __dadd_rn(s1, s2);
     S.xm[k] = __double_as_longlong(s1) >= __double_as_longlong(s2) ? S.x1[k] : S.x2[k];
+#elif EP_T_FMA
+    S.t[k] = fma(S.x1[k], S.x1[k], __dmul_rn(S.x2[k], S.x2[k]));
 #else
     S.t[k] = __dadd_rn(__dmul_rn(S.x1[k], S.x1[k]), __dmul_rn(S.x2[k], S.x2[k]));
 #endif
@@ -535,15 +560,23 @@ __device__ __forceinline__ void gen_stage(unsigned& vlo, unsigned& vhi, const EP
 template <int W, bool DBG = false>
 __device__ __forceinline__ void transform_stage(const Stage<W>& S, const EPParams& P, const LeanConst& K,
                                                 PairAcc& A, unsigned long long* s_rare,
-                                                double* dbg = nullptr) {
+                                                double* dbg = nullptr, unsigned nvalid = W) {
   double r[W], c[W], L[W], p[W], y0[W], e[W], g[W], t2[W], X[W], Y[W];
   unsigned l[W];
-  bool acc[W], ok[W];
+  bool acc[W], ok[W], band[W];
 #pragma unroll
   for (int k = 0; k < W; ++k) {
-    if (EP_PRED_MODE == 1 && !DBG)
-      acc[k] = true;  // decided by the selector below (rejects -> NaN or >= 2^21)
-    else if (EP_ACC_HI && !DBG)
+    band[k] = false;
+    if (EP_T_FMA == 1) {
+      // t' is the fused t' (<= 1 ulp from NPB's): settled on the fast path
+      // only below the high word 0x3FCFFFFF; the two high words around 1/4
+      // (P ~ 1e-6 per pair) go to the rare path, which decides exactly
+      const unsigned h = static_cast<unsigned>(__double2hiint(S.t[k]));
+      acc[k] = h < 0x3FCFFFFFu;
+      band[k] = h - 0x3FCFFFFFu <= 1u;
+    } else if (EP_PRED_MODE == 1 && !DBG)
+      acc[k] = k < nvalid;  // decided by the selector below (rejects -> NaN or >= 2^21)
+    else if (EP_ACC_HI && (!DBG || EP_T_FMA == 2))
       // high word only: t' < 1/4 is decided exactly; hi == bits(1/4) holds
       // t' == 1/4 (L = 0 -> X = Y = 0, bin 0: correct on the fast path) and
       // rejects just above 1/4, whose L < 0 makes X, Y NaN -> selector says
@@ -553,8 +586,12 @@ __device__ __forceinline__ void transform_stage(const Stage<W>& S, const EPParam
       acc[k] = static_cast<unsigned long long>(__double_as_longlong(S.t[k])) <= 0x3FD0000000000000ull;
     else
       acc[k] = S.t[k] <= 0.25;
+    if (EP_T_FMA == 1) band[k] = band[k] && k < nvalid;
+    acc[k] = acc[k] && k < nvalid;  // (nvalid < W only in a thread's last, partial group)
     r[k] = fma(S.t[k], S.eInv[k], -1.0);
-#if EP_LOG_K >= 9
+#if EP_LOG_DEG4 && EP_LOG_K >= 9
+    c[k] = fma(r[k], 0.5, P.coef[2]);  // -2 ln(1+r) = r(-2 + r(1 + r(-2/3 + r/2))) + O(r^5)
+#elif EP_LOG_K >= 9
     c[k] = fma(r[k], K.c6, 0.5);  // K.c6 holds c5 = -2/5 (20-bit) for the degree-5 series
 #elif EP_KMODE == 1
     c[k] = fma(r[k], EP_C6, P.coef[1]);  // c6 immediate (b slot), c5 uniform (param -> UR)
@@ -568,8 +605,10 @@ __device__ __forceinline__ void transform_stage(const Stage<W>& S, const EPParam
 #pragma unroll
   for (int k = 0; k < W; ++k) c[k] = fma(c[k], r[k], 0.5);
 #endif
+#if !(EP_LOG_DEG4 && EP_LOG_K >= 9)
 #pragma unroll
   for (int k = 0; k < W; ++k) c[k] = fma(c[k], r[k], P.coef[2]);
+#endif
 #pragma unroll
   for (int k = 0; k < W; ++k) c[k] = fma(c[k], r[k], 1.0);
 #pragma unroll
@@ -651,17 +690,19 @@ __device__ __forceinline__ void transform_stage(const Stage<W>& S, const EPParam
       A.cnt += bin_increment(l[k], K.one);
     }
 #if EP_PRED_MODE != 1
-    any_rare |= acc[k] && !ok[k];
+    any_rare |= (acc[k] && !ok[k]) || band[k];
 #endif
     if (DBG && EP_MAXSQ) {
       X[k] = __dmul_rn(S.x1[k], t2[k]);
       Y[k] = __dmul_rn(S.x2[k], t2[k]);
     }
     if (DBG) {  // test hook (hpl_ep_pairs_debug): t, X, Y, l (-1 rare path, -2 rejected)
-      dbg[4 * k + 0] = 4.0 * S.t[k];
+      // t as NPB rounds it (the fused t' of EP_T_FMA is internal)
+      dbg[4 * k + 0] = 4.0 * __dadd_rn(__dmul_rn(S.x1[k], S.x1[k]), __dmul_rn(S.x2[k], S.x2[k]));
       dbg[4 * k + 1] = ok[k] ? X[k] : 0.0;
       dbg[4 * k + 2] = ok[k] ? Y[k] : 0.0;
-      dbg[4 * k + 3] = ok[k] ? double(EP_BIN_MODE == 3 ? l[k] & 3u : l[k]) : (acc[k] ? -1.0 : -2.0);
+      const bool acc_npb = __dadd_rn(__dmul_rn(S.x1[k], S.x1[k]), __dmul_rn(S.x2[k], S.x2[k])) <= 0.25;
+      dbg[4 * k + 3] = !acc_npb ? -2.0 : ok[k] ? double(EP_BIN_MODE == 3 ? l[k] & 3u : l[k]) : -1.0;
     }
   }
 #if EP_PRED_MODE == 1
@@ -674,7 +715,7 @@ __device__ __forceinline__ void transform_stage(const Stage<W>& S, const EPParam
 #endif
 #pragma unroll
     for (int k = 0; k < W; ++k)
-      if (EP_PRED_MODE == 1 ? (l[k] - 0x49800004u < 0x007FFFFCu) : (acc[k] && !ok[k])) {
+      if (EP_PRED_MODE == 1 ? (l[k] - 0x49800004u < 0x007FFFFCu) : ((acc[k] && !ok[k]) || band[k])) {
         if (EP_MAXSQ) {
           X[k] = __dmul_rn(S.x1[k], t2[k]);
           Y[k] = __dmul_rn(S.x2[k], t2[k]);
@@ -744,6 +785,82 @@ __device__ __forceinline__ void libdevice_pair(unsigned& vlo, unsigned& vhi, con
   }
 }
 
+// The pipelined pair loop of one thread (A3-A7): `iters` full iterations of
+// PER_IT pairs, then the last `tail` (<= PER_IT) pairs with the rest of the
+// group masked.  Out of line (EP_LOOP_NOINLINE) so that ptxas allocates and
+// schedules the hot loop on its own, independent of the kernel's prologue
+// (skip-ahead, table copy) and epilogue (reduction, combine).
+struct LoopOut {
+  double sx, sy;
+  unsigned q0, q1, q2, q3;
+};
+#ifndef EP_LOOP_NOINLINE
+#define EP_LOOP_NOINLINE 0
+#endif
+#if EP_LOOP_NOINLINE
+#define EP_LOOP_INL __noinline__
+#else
+#define EP_LOOP_INL __forceinline__
+#endif
+template <bool A32, int W>
+__device__ EP_LOOP_INL LoopOut pair_loop(unsigned vlo, unsigned vhi, uint64_t n_t, const EPParams& P, unsigned tab,
+                                         unsigned kc, unsigned long long* s_rare) {
+  double sx = 0.0, sy = 0.0;
+  unsigned q0 = 0, q1 = 0, q2 = 0, q3 = 0;
+  auto flush = [&](const PairAcc& A) {
+    q0 += A.cnt & 0xFFu;
+    q1 += (A.cnt >> 8) & 0xFFu;
+    q2 += (A.cnt >> 16) & 0xFFu;
+    q3 += A.cnt >> 24;
+    sx += A.csx;
+    sy += A.csy;
+  };
+  {
+    // 8-bit packed counters overflow after 255 pairs: <= 252 pairs per flush.
+    constexpr unsigned PER_IT = (EP_PIPE_ORDER == 1 ? 1 : 2) * W, IT_PER_CHUNK = 252 / PER_IT;
+    // Warp-uniform trip count: every thread runs base / PER_IT pipelined
+    // iterations (base = the grid-wide floor); the rest (<= PER_IT pairs)
+    // goes through the same stages once more with the pairs past the
+    // thread's range masked out (the loop's one-group overshoot is exactly
+    // the next group of the stream).
+    const unsigned tail = unsigned(n_t - (P.base / PER_IT) * PER_IT);
+    uint64_t iters = P.base / PER_IT;
+    const LeanConst K = make_lean_const(kc);
+    Stage<W> s0, s1;
+    gen_stage<A32, W>(vlo, vhi, P, tab, s0, K.exp_hi);
+    while (iters) {
+      const unsigned ci = iters < IT_PER_CHUNK ? unsigned(iters) : IT_PER_CHUNK;
+      PairAcc A{0.0, 0.0, 0u};
+#pragma unroll kLoopUnroll
+      for (unsigned i = 0; i < ci; ++i) {
+#if EP_PIPE_ORDER == 1
+        transform_stage<W>(s0, P, K, A, s_rare);
+        gen_stage<A32, W>(vlo, vhi, P, tab, s0, K.exp_hi);
+        (void)s1;
+#else
+        gen_stage<A32, W>(vlo, vhi, P, tab, s1, K.exp_hi);
+        transform_stage<W>(s0, P, K, A, s_rare);
+        gen_stage<A32, W>(vlo, vhi, P, tab, s0, K.exp_hi);
+        transform_stage<W>(s1, P, K, A, s_rare);
+#endif
+      }
+      flush(A);
+      iters -= ci;
+    }
+    // the thread's last <= PER_IT pairs: s0 already holds the next group
+    if (__any_sync(0xFFFFFFFFu, tail != 0)) {
+      PairAcc A{0.0, 0.0, 0u};
+      transform_stage<W>(s0, P, K, A, s_rare, nullptr, tail < W ? tail : W);
+#if EP_PIPE_ORDER != 1
+      gen_stage<A32, W>(vlo, vhi, P, tab, s1, K.exp_hi);
+      transform_stage<W>(s1, P, K, A, s_rare, nullptr, tail > W ? tail - W : 0u);
+#endif
+      flush(A);
+    }
+  }
+  return LoopOut{sx, sy, q0, q1, q2, q3};
+}
+
 template <int VARIANT, bool A32, int NT, int MINB, int W>
 __global__ void __launch_bounds__(NT, MINB)
 ep_kernel(const __grid_constant__ EPParams P) {
@@ -781,7 +898,7 @@ ep_kernel(const __grid_constant__ EPParams P) {
         if (i0 + k * nt < LOG_TAB) dst[i0 + k * nt] = v[k];
     }
   }
-  if (VARIANT == HPL_VARIANT_LEAN && EP_TMA_TABLE && tid == 0) {
+  if (VARIANT == HPL_VARIANT_LEAN && EP_TMA_TABLE && !(EP_ABL & 64) && tid == 0) {
     constexpr unsigned BYTES = LOG_TAB * sizeof(LogEntry), CHUNK = 32768;
     asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(mbar));
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -795,6 +912,21 @@ ep_kernel(const __grid_constant__ EPParams P) {
                    ::"r"(dst + off), "l"(src + off), "r"(n), "r"(mbar) : "memory");
     }
   }
+#if EP_JUMP_WIN
+  // A2 skip-ahead by 4-bit windows: s_win[i][d] = a^(d 16^i) mod 2^46 from the
+  // binary jump table (<= 4 mulmods per entry, one entry per thread), so each
+  // thread's jump below is <= 12 table multiplies instead of up to 46
+  // predicated ones (~1 us less per launch; DESIGN.md §6 fixed cost)
+  __shared__ uint64_t s_win[EP_WIN_N][16];
+  for (unsigned e = tid; e < EP_WIN_N * 16; e += blockDim.x) {
+    const unsigned wi = e >> 4, d = e & 15;
+    uint64_t w = 1;
+#pragma unroll
+    for (unsigned b = 0; b < 4; ++b)
+      if (((d >> b) & 1) && 4 * wi + b < NJUMP) w = mulmod46(w, P.jump[4 * wi + b]);
+    s_win[wi][d] = w;
+  }
+#endif
   if (tid < 7) s_rare[tid] = 0;
   if (tid == 0) {
     s_kc[0] = EP_LOG_K >= 9 ? EP_C5 : EP_C6;
@@ -817,11 +949,21 @@ ep_kernel(const __grid_constant__ EPParams P) {
   const uint64_t gid = uint64_t(blockIdx.x) * blockDim.x + tid;
   const uint64_t n_t = P.base + (gid < P.extra ? 1 : 0);
   const uint64_t p0 = gid * P.base + (gid < P.extra ? gid : P.extra);
+#if EP_ABL & 128  // ablation: no skip-ahead
+  const uint64_t v0 = state_to_v(P.x_begin + 2 * p0);
+#elif EP_JUMP_WIN
+  uint64_t xj = P.x_begin;
+#pragma unroll 1
+  for (uint64_t k = 2 * p0, wi = 0; k != 0; k >>= 4, ++wi)
+    if (k & 15) xj = mulmod46(xj, s_win[wi][k & 15]);
+  const uint64_t v0 = state_to_v(xj);
+#else
   const uint64_t v0 = state_to_v(jump_state(P.x_begin, 2 * p0, P.jump));
+#endif
   unsigned vlo = unsigned(v0), vhi = unsigned(v0 >> 32);
 #if EP_TMA_WAIT_LATE
   // the skip-ahead above overlapped the table's bulk copy; wait for it now
-  if (VARIANT == HPL_VARIANT_LEAN && EP_TMA_TABLE) {
+  if (VARIANT == HPL_VARIANT_LEAN && EP_TMA_TABLE && !(EP_ABL & 64)) {
     unsigned done = 0;
     while (!done)
       asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], 0;\n\t"
@@ -839,44 +981,17 @@ ep_kernel(const __grid_constant__ EPParams P) {
     sx += A.csx;
     sy += A.csy;
   };
-  if (VARIANT == HPL_VARIANT_LEAN && EP_PIPE) {
-    // 8-bit packed counters overflow after 255 pairs: <= 252 pairs per flush.
-    // Tail pairs first, so the pipelined loop's one-group overshoot past the
-    // thread's range is never transformed.
-    constexpr unsigned PER_IT = (EP_PIPE_ORDER == 1 ? 1 : 2) * W, IT_PER_CHUNK = 252 / PER_IT;
-    // Warp-uniform trip count: every thread runs base / PER_IT pipelined
-    // iterations (base = the grid-wide floor), the rest (< PER_IT + 1 pairs)
-    // goes through the tail loop.
-    const unsigned tail = unsigned(n_t - (P.base / PER_IT) * PER_IT);
-    if (tail) {
-      PairAcc A{0.0, 0.0, 0u};
-#pragma unroll 1
-      for (unsigned i = 0; i < tail; ++i) lean_pair<A32>(vlo, vhi, P, tab, A, s_rare);
-      flush(A);
-    }
-    uint64_t iters = P.base / PER_IT;
-    const LeanConst K = make_lean_const(static_cast<unsigned>(__cvta_generic_to_shared(s_kc)));
-    Stage<W> s0, s1;
-    if (iters) gen_stage<A32, W>(vlo, vhi, P, tab, s0, K.exp_hi);
-    while (iters) {
-      const unsigned ci = iters < IT_PER_CHUNK ? unsigned(iters) : IT_PER_CHUNK;
-      PairAcc A{0.0, 0.0, 0u};
-#pragma unroll kLoopUnroll
-      for (unsigned i = 0; i < ci; ++i) {
-#if EP_PIPE_ORDER == 1
-        transform_stage<W>(s0, P, K, A, s_rare);
-        gen_stage<A32, W>(vlo, vhi, P, tab, s0, K.exp_hi);
-        (void)s1;
-#else
-        gen_stage<A32, W>(vlo, vhi, P, tab, s1, K.exp_hi);
-        transform_stage<W>(s0, P, K, A, s_rare);
-        gen_stage<A32, W>(vlo, vhi, P, tab, s0, K.exp_hi);
-        transform_stage<W>(s1, P, K, A, s_rare);
-#endif
-      }
-      flush(A);
-      iters -= ci;
-    }
+  if (EP_ABL & 32) {  // ablation: no pairs (fixed cost only)
+    sx = double(vlo); sy = double(vhi);
+  } else if (VARIANT == HPL_VARIANT_LEAN && EP_PIPE) {
+    const LoopOut o = pair_loop<A32, W>(vlo, vhi, n_t, P, tab, static_cast<unsigned>(__cvta_generic_to_shared(s_kc)),
+                                        s_rare);
+    sx = o.sx;
+    sy = o.sy;
+    q0 = o.q0;
+    q1 = o.q1;
+    q2 = o.q2;
+    q3 = o.q3;
   } else {
     // 8-bit packed counters overflow after 255 pairs: chunks of 252 = 63 x 4
     constexpr unsigned UNROLL = 4, CHUNK = 63 * UNROLL;
@@ -928,53 +1043,90 @@ ep_kernel(const __grid_constant__ EPParams P) {
     s_wq[warp][3] = w3;
   }
   __syncthreads();
-  if (tid == 0) {
-    EPPartial part;
-    part.sx = 0.0;
-    part.sy = 0.0;
-    for (int k = 0; k < 4; ++k) part.q[k] = 0;
+  if (warp == 0) {  // warp 0 folds the per-warp values by a fixed shuffle tree
     const unsigned nw = blockDim.x >> 5;
-    for (unsigned w = 0; w < nw; ++w) {
-      part.sx += s_wsx[w];
-      part.sy += s_wsy[w];
-      for (int k = 0; k < 4; ++k) part.q[k] += s_wq[w][k];
+    double a = 0.0, b = 0.0;
+    unsigned long long c[4] = {0, 0, 0, 0};
+    for (unsigned w = lane; w < nw; w += 32) {
+      a += s_wsx[w];
+      b += s_wsy[w];
+      for (int k = 0; k < 4; ++k) c[k] += s_wq[w][k];
     }
-    for (int k = 4; k < 10; ++k) part.q[k] = s_rare[k - 4];
-    part.big = s_rare[6];
-    P.partials[blockIdx.x] = part;
-    __threadfence();
-    const unsigned ticket = atomicAdd(P.counter, 1u);
-    s_last = (ticket == gridDim.x - 1);
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) {
+      a += __shfl_xor_sync(0xFFFFFFFFu, a, off);
+      b += __shfl_xor_sync(0xFFFFFFFFu, b, off);
+#pragma unroll
+      for (int k = 0; k < 4; ++k) c[k] += __shfl_xor_sync(0xFFFFFFFFu, c[k], off);
+    }
+    if (lane == 0) {
+      EPPartial part;
+      part.sx = a;
+      part.sy = b;
+      for (int k = 0; k < 4; ++k) part.q[k] = c[k];
+      for (int k = 4; k < 10; ++k) part.q[k] = s_rare[k - 4];
+      part.big = s_rare[6];
+      P.partials[blockIdx.x] = part;
+      __threadfence();
+      const unsigned ticket = atomicAdd(P.counter, 1u);
+      s_last = (ticket == gridDim.x - 1);
+    }
   }
   __syncthreads();
-  if (!s_last) return;
+  if (!s_last || (EP_ABL & 256)) return;  // (ablation 256: no last-block fold)
   // last block: 16-thread groups; thread (group gi, word w) folds word w of
   // partials gi, gi + ng, ... (independent loads in flight), then thread w
   // folds the groups in order — fixed order, so bitwise deterministic.
   __threadfence();
   {
     const unsigned G = gridDim.x, ng = blockDim.x >> 4, gi = tid >> 4, w = tid & 15;
+    // FOLD_U loads issued before the first add: one L2 round trip per FOLD_U
+    // partials instead of one per partial (same summation order)
+    constexpr unsigned FOLD_U = 8;
     if (w < 13) {
       if (w < 2) {
         double sacc = 0.0;
-        for (unsigned b = gi; b < G; b += ng) sacc += __ldcg(w == 0 ? &P.partials[b].sx : &P.partials[b].sy);
+        for (unsigned b0 = gi; b0 < G; b0 += FOLD_U * ng) {
+          double v[FOLD_U];
+#pragma unroll
+          for (unsigned k = 0; k < FOLD_U; ++k) {
+            const unsigned b = b0 + k * ng;
+            v[k] = b < G ? __ldcg(w == 0 ? &P.partials[b].sx : &P.partials[b].sy) : 0.0;
+          }
+#pragma unroll
+          for (unsigned k = 0; k < FOLD_U; ++k) sacc += v[k];
+        }
         s_fold[gi][w] = __double_as_longlong(sacc);
       } else {
         unsigned long long sacc = 0;
-        for (unsigned b = gi; b < G; b += ng) sacc += __ldcg(w < 12 ? &P.partials[b].q[w - 2] : &P.partials[b].big);
+        for (unsigned b0 = gi; b0 < G; b0 += FOLD_U * ng) {
+          unsigned long long v[FOLD_U];
+#pragma unroll
+          for (unsigned k = 0; k < FOLD_U; ++k) {
+            const unsigned b = b0 + k * ng;
+            v[k] = b < G ? __ldcg(w < 12 ? &P.partials[b].q[w - 2] : &P.partials[b].big) : 0ull;
+          }
+#pragma unroll
+          for (unsigned k = 0; k < FOLD_U; ++k) sacc += v[k];
+        }
         s_fold[gi][w] = static_cast<long long>(sacc);
       }
     }
     __syncthreads();
-    if (tid < 13) {
-      if (tid < 2) {
+    // warp j folds word j over the groups: lane-strided, then a fixed shuffle tree
+    for (unsigned word = warp; word < 13; word += blockDim.x >> 5) {
+      if (word < 2) {
         double sacc = 0.0;
-        for (unsigned g = 0; g < ng; ++g) sacc += __longlong_as_double(s_fold[g][tid]);
-        s_fin[tid] = sacc;
+        for (unsigned g = lane; g < ng; g += 32) sacc += __longlong_as_double(s_fold[g][word]);
+#pragma unroll
+        for (int off = 16; off > 0; off >>= 1) sacc += __shfl_xor_sync(0xFFFFFFFFu, sacc, off);
+        if (lane == 0) s_fin[word] = sacc;
       } else {
         unsigned long long sacc = 0;
-        for (unsigned g = 0; g < ng; ++g) sacc += static_cast<unsigned long long>(s_fold[g][tid]);
-        s_fin[tid] = static_cast<double>(sacc);  // exact: < 2^53
+        for (unsigned g = lane; g < ng; g += 32) sacc += static_cast<unsigned long long>(s_fold[g][word]);
+#pragma unroll
+        for (int off = 16; off > 0; off >>= 1) sacc += __shfl_xor_sync(0xFFFFFFFFu, sacc, off);
+        if (lane == 0) s_fin[word] = static_cast<double>(sacc);  // exact: < 2^53
       }
     }
   }
@@ -1160,6 +1312,9 @@ void build_log_table(std::vector<LogEntry>& tab) {
       const float inv = (float)(1.0L / centre);
       tab[e].inv = (double)inv;
       tab[e].T = (double)(2.0L * logl((long double)inv * 0.25L));  // -2 ln(4 t') at r = 0
+    } else if (EP_T_FMA == 2 && j == LOG_IDX_MAX) {  // [1/4, 1/4 + w) and, via the H + 1 index,
+      tab[e].T = __builtin_nan("");                  // the fused t' just below 1/4: NaN -> the
+      tab[e].inv = __builtin_nan("");                // rare path decides acceptance on NPB's t'
     } else if (j <= LOG_IDX_MAX) {      // [1/4 - w, 1/4 + w), reference point 1/4 itself (T = 0,
                                         // r = 4t' - 1 exact): L = -2 ln(1 + r) has no cancellation
                                         // as t' -> 1/4; t' = 1/4 -> L = 0; above -> L < 0 -> NaN

@@ -30,7 +30,9 @@ for ln in out.splitlines():
 best = None
 for addr, i in ins:
     m = re.search(r"BRA (?:!?U?P\d, )?0x([0-9a-f]+)", i)
-    if m and int(m.group(1), 16) < addr:
+    # the loop's back edge is conditional (@P BRA); unconditional backward
+    # branches are the rare paths' returns into the loop body
+    if m and int(m.group(1), 16) < addr and i.startswith("@"):
         lo = int(m.group(1), 16)
         n = sum(1 for a, j in ins if lo <= a <= addr and "RSQ64H" in j)
         # the pipelined group loop holds exactly one MUFU per pair of an
