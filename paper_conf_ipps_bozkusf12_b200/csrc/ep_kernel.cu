@@ -46,6 +46,10 @@ __device__ __forceinline__ double rsqrt_approx(double p) {
   return y;
 }
 
+#ifndef EP_T_FMA
+#define EP_T_FMA 2     // t' = fma(x1', x1', RN(x2'^2)) (one DADD less; |t'_f - t'| <= 1.5 2^-52 t', DESIGN R11);
+#endif                 // 2: the fused t' just below 1/4 indexes the NaN bucket -> rare path, which recomputes
+                       //    NPB's t' and decides acceptance exactly; 1: same by an explicit band test
 #ifndef EP_IDX_TRUNC
 #define EP_IDX_TRUNC 1  // 1: truncating table index (VIMNMX + SHF + LEA; ep_common.cuh)
 #endif
@@ -424,7 +428,7 @@ __device__ __forceinline__ void lean_pairs(unsigned& vlo, unsigned& vhi, const E
 }
 
 #ifndef EP_LOOP_UNROLL
-#define EP_LOOP_UNROLL 1  // unroll of the pipelined group loop (codegen/register-allocation knob)
+#define EP_LOOP_UNROLL 2  // unroll of the pipelined group loop (codegen/register-allocation knob; 2: +1.6 % with EP_T_FMA 2)
 #endif
 constexpr int kLoopUnroll = EP_LOOP_UNROLL;  // (#pragma arguments are not macro-expanded)
 #ifndef EP_PIPE_ORDER
@@ -470,9 +474,6 @@ constexpr int kLoopUnroll = EP_LOOP_UNROLL;  // (#pragma arguments are not macro
 #ifndef EP_LOG_DEG4
 #define EP_LOG_DEG4 1  // 1: degree-4 series for -2 ln(1+r) (K >= 9: |error| <= (2/5) 2^-50 absolute in L)
 #endif
-#ifndef EP_T_FMA
-#define EP_T_FMA 0     // 1: t' = fma(x1', x1', RN(x2'^2)) (<= 1 ulp from NPB's t'); t' within 2^-20 of 1/4
-#endif                 //    goes to the rare path, which recomputes NPB's t' and decides acceptance exactly
 #ifndef EP_JUMP_WIN
 #define EP_JUMP_WIN 1  // 1: per-thread skip-ahead by 4-bit windows (shared-memory table)
 #endif
@@ -1077,7 +1078,13 @@ ep_kernel(const __grid_constant__ EPParams P) {
   // last block: 16-thread groups; thread (group gi, word w) folds word w of
   // partials gi, gi + ng, ... (independent loads in flight), then thread w
   // folds the groups in order — fixed order, so bitwise deterministic.
+#if !(EP_ABL & 512)  // (ablation 512: no fence before the fold)
   __threadfence();
+#endif
+#if EP_ABL & 1024  // ablation: fold without reading the partials
+  if (tid < 13) s_fin[tid] = double(tid);
+  if (false)
+#endif
   {
     const unsigned G = gridDim.x, ng = blockDim.x >> 4, gi = tid >> 4, w = tid & 15;
     // FOLD_U loads issued before the first add: one L2 round trip per FOLD_U

@@ -150,6 +150,15 @@ def gpu_range(gpu, seed, a, begin, n, threads=0):
     return hpl.unpack13(out.cpu().tolist())
 
 
+def dev_tol(Xe, Ye):
+    """|X - X_exact| allowed for the kernel: 4 ulp (table log, Newton, products)
+    plus the fused t' (DESIGN R11): |dX| <= |X| (1/L + 1/2) 1.5 2^-52, L = X^2 + Y^2
+    (the series term is < 2^-50 |X|/L, covered by the same slack)."""
+    L = float(Xe) ** 2 + float(Ye) ** 2
+    f = (1.0 / L + 0.5) * 1.5 * 2.0 ** -52 if L > 0 else 0.0
+    return (4 * math.ulp(float(Xe)) + abs(float(Xe)) * f, 4 * math.ulp(float(Ye)) + abs(float(Ye)) * f)
+
+
 def gpu_pair(gpu, seed, a):
     _, hpl = gpu
     return np.frombuffer(hpl.hpl_ep_pairs_debug(seed, a, 0, 1), dtype=np.float64).reshape(1, 4)[0]
@@ -175,10 +184,14 @@ def test_gpu_t_cases(gpu, oracle_mod, name, threads):
     if name == "t_above_1":
         assert l == -2
     elif name == "t_eq_1":
-        assert (X, Y, l) == (0.0, 0.0, 0.0)          # fast path: L = 0, t2 = 0
+        # L = 0, t2 = 0, X = Y = 0, bin 0 — settled by the rare path (-1), which
+        # recomputes NPB's t for every fused t' next to 1/4 (R11), or by the
+        # fast path (0) in builds without the fused t'
+        assert X == 0.0 and Y == 0.0 and l in (0.0, -1.0)
     else:
         _, Xe, Ye = exact_m(k1, k2)
-        assert abs(X - float(Xe)) <= 4 * math.ulp(float(Xe)) and abs(Y - float(Ye)) <= 4 * math.ulp(float(Ye))
+        tx, ty = dev_tol(Xe, Ye)
+        assert abs(X - float(Xe)) <= tx and abs(Y - float(Ye)) <= ty
 
 
 @pytest.mark.gpu
@@ -187,7 +200,8 @@ def test_gpu_m_cases(gpu, oracle_mod, key):
     """Bin boundaries 1..4: 8-16 ulp away the GPU bin equals the exact (and the
     oracle's) bin; within ~1 ulp the GPU's bin is trunc of its own
     max(|X|,|Y|) (the FP32-view selector / rare-path split is exact) and its
-    X, Y are within 4 ulp of the exact deviates."""
+    X, Y are within dev_tol of the exact deviates (<= 6.25 ulp at M >= 1,
+    since L >= M^2)."""
     K, tag = key
     k1, k2 = M_CASES[key]
     seed, a = stream_for(k1, k2)
@@ -196,7 +210,8 @@ def test_gpu_m_cases(gpu, oracle_mod, key):
     assert g["gc"] == 1
     lg = g["q"].index(1)
     X, Y = g["sx"], g["sy"]
-    assert abs(X - float(Xe)) <= 4 * math.ulp(float(Xe)) and abs(Y - float(Ye)) <= 4 * math.ulp(float(Ye))
+    tx, ty = dev_tol(Xe, Ye)
+    assert abs(X - float(Xe)) <= tx and abs(Y - float(Ye)) <= ty
     assert lg == int(max(abs(X), abs(Y)))
     if tag in ("m12", "p12"):
         assert lg == int(m)

@@ -5,10 +5,16 @@ individual pairs; here every pair is compared with an independent reference:
 the LCG states from the oracle's randlc, NPB's t = RN(RN(x1²)+RN(x2²)) in IEEE
 double (numpy never fuses), and X, Y = x·sqrt(-2 ln t / t) in 80-bit long
 double.  Claims pinned: acceptance decisions exact; |X - X_true| <= 4 ulp of
-X plus the degree-4 log series' truncation |dL| <= (2/5) 2^-50 carried into X
-(dX = X dL / 2L: below one ulp wherever L >= 1, i.e. for every
-pair whose max(|X|,|Y|) can reach a bin boundary); bins equal
-trunc(max(|X_true|,|Y_true|)); no systematic bias.
+X plus two derived terms (reading R11):
+  * the degree-4 log series' truncation |dL| <= (2/5) 2^-50, carried into X
+    as dX = X dL / 2L;
+  * the fused t' = fma(x1', x1', RN(x2'^2)) of the hot loop, which differs from
+    NPB's t' by |dt| <= 1.5 2^-52 t, carried into X as |dX/X| <= (1/L + 1/2) dt/t
+    (X = x sqrt(L/t), dL = -2 dt/t);
+both below 4.5 ulp wherever L >= 1, i.e. for every pair whose max(|X|,|Y|) can
+reach a bin boundary (the oracle's bin margin is >= 8627 ulp at class D, R7);
+bins equal trunc(max(|X_true|,|Y_true|)); no systematic bias.  t == 1 and the
+other constructed boundary pairs are in tests/test_edge_pairs.py.
 """
 import numpy as np
 import pytest
@@ -51,9 +57,16 @@ def reference(oracle_mod, seed, a, begin, n):
 DL_SERIES = 1.05 * 0.4 * 2.0 ** -50
 
 
+# |t'_fused - t'_NPB| / t' (one rounding of x1'^2 skipped, one sum rounding)
+DT_FMA = 1.5 * 2.0 ** -52
+
+
 def tolerance_ulps(Xr, L, ulp):
-    """4 ulp of rounding + the series truncation carried into X (dX = X dL/2L)."""
-    return 4.0 + (np.abs(Xr) * DL_SERIES / (2.0 * L)).astype(np.float64) / ulp
+    """4 ulp of rounding + the series truncation (dX = X dL/2L) + the fused t'
+    (|dX| <= |X| (1/L + 1/2) dt/t)."""
+    Xa = np.abs(Xr)
+    extra = Xa * DL_SERIES / (2.0 * L) + Xa * (1.0 / L + 0.5) * DT_FMA
+    return 4.0 + extra.astype(np.float64) / ulp
 
 
 @pytest.mark.parametrize("seed,begin", [(NPB_SEED, 0), (NPB_SEED, 2 ** 36 - 2 ** 21), (1, 12345), ((1 << 46) - 1, 999)])
@@ -71,9 +84,9 @@ def test_per_pair_accuracy(hpl, oracle_mod, seed, begin):
     assert np.all(eX <= tolerance_ulps(Xr[a], L[a], ulp(Xr[a])))
     assert np.all(eY <= tolerance_ulps(Yr[a], L[a], ulp(Yr[a])))
     # where bins can change (L >= 1: max(|X|,|Y|) >= 1 needs L >= t/x^2 >= 1)
-    # the plain 4-ulp bound holds
+    # the error stays below 4 + 1.5 * 1.5 * 2 = 8.5 ulp
     big = a & (L >= 1)
-    assert float(np.max(np.abs(gX[big] - Xr[big]) / ulp(Xr[big]))) <= 4.0
+    assert float(np.max(np.abs(gX[big] - Xr[big]) / ulp(Xr[big]))) <= 8.5
     # no systematic bias: mean signed error well below one ulp where the
     # rounding dominates, and the absolute error of the sums' terms averages out
     sX = (gX[big] - Xr[big]) / ulp(Xr[big])
@@ -86,17 +99,10 @@ def test_per_pair_accuracy(hpl, oracle_mod, seed, begin):
     assert np.array_equal(gl[fast].astype(np.int64), lt[fast])
     # the rare path takes exactly the l >= 4 pairs and those below the table
     rare = gl == -1
-    assert np.all((lt[rare] >= 4) | (t[rare] < 2.0 ** -16 * 1.01))
+    # (and, with the fused t', those whose t is within a few ulp below 1: the
+    # rare path settles their acceptance on NPB's t)
+    assert np.all((lt[rare] >= 4) | (t[rare] < 2.0 ** -16 * 1.01) | (t[rare] >= 1.0 - 2.0 ** -19))
     assert np.all(lt[fast] < 4)
-
-
-def test_exact_boundary_t_equals_one(hpl):
-    """t == 1 gives L = 0, t2 = 0, X = Y = 0, bin 0 (reading R5) — checked on
-    whatever pairs of a long stretch land there, and on the decision logic."""
-    n = 1 << 20
-    out = np.frombuffer(hpl.hpl_ep_pairs_debug(NPB_SEED, NPB_A, 777, n), dtype=np.float64).reshape(n, 4)
-    one = out[:, 0] == 1.0
-    assert np.all(out[one, 1] == 0.0) and np.all(out[one, 3] == 0.0)
 
 
 def test_worked_example_first_pairs(hpl):
@@ -107,5 +113,8 @@ def test_worked_example_first_pairs(hpl):
     out = np.frombuffer(hpl.hpl_ep_pairs_debug(NPB_SEED, NPB_A, 0, len(rows)), dtype=np.float64).reshape(-1, 4)
     for r, o in zip(rows, out):
         X, Y = float(r[1]), float(r[2])
-        assert abs(o[1] - X) <= 4 * np.spacing(abs(X)) and abs(o[2] - Y) <= 4 * np.spacing(abs(Y))
+        # 4 ulp (kernel) + 1 (the fixture's glibc) + the fused t' term 3 (1/L + 1/2)
+        # ulp; L = X^2 + Y^2 (X^2 + Y^2 = t L / t)
+        tol = 5 + 3 * (1 / (X * X + Y * Y) + 0.5)
+        assert abs(o[1] - X) <= tol * np.spacing(abs(X)) and abs(o[2] - Y) <= tol * np.spacing(abs(Y))
         assert int(o[3]) == int(r[3])

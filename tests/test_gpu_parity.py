@@ -288,6 +288,33 @@ def test_npb_class_E_verification_sums(env):
     assert q[9] == 0 and q[8] <= 2
 
 
+def test_class_E_sampled_ranges(env, oracle_mod):
+    """Class E q[] parity where the oracle can follow: sampled sub-ranges of the
+    M = 40 stream (incl. the first pairs and the last ones before 2^40) through
+    the same kernel, q and gc exact, sums within T1."""
+    rng = random.Random(40)
+    for begin in [0, 2 ** 40 - 2 ** 21] + [rng.randrange(2 ** 40 - 2 ** 21) for _ in range(3)]:
+        g = gpu_range(env, NPB_SEED, NPB_A, begin, 2 ** 21)
+        assert_parity(g, oracle_mod.run_pairs(NPB_SEED, NPB_A, begin, 2 ** 21))
+
+
+def test_class_E_shards_add_up(env):
+    """Class E split into 8 shards (the 8-GPU layout, run serially here): the
+    shards' q and gc add up to the whole run's bit for bit, sums within T1."""
+    torch, hpl = env
+    M = 40
+    sx, sy, q = hpl.hpl_ep_run(M, NPB_SEED, NPB_A)
+    acc = torch.zeros(13, dtype=torch.float64, device="cuda")
+    for r in range(8):
+        out = torch.empty(13, dtype=torch.float64, device="cuda")
+        hpl.hpl_ep_run_shard(M, NPB_SEED, NPB_A, r, 8, out.data_ptr(), torch.cuda.current_stream().cuda_stream)
+        acc += out
+    torch.cuda.synchronize()
+    g = hpl.unpack13(acc.cpu().tolist())
+    assert g["q"] == list(q) and g["gc"] == sum(q)
+    assert sums_close(g["sx"], sx, sum(q)) and sums_close(g["sy"], sy, sum(q))
+
+
 @pytest.mark.parametrize("case", range(8))
 def test_random_streams(env, oracle_mod, case):
     """Seeded random (seed, a, range) combinations incl. wide multipliers and

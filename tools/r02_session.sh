@@ -1,0 +1,39 @@
+#!/bin/bash
+# Round-2 GPU session (under gpurun): tests + bench of the default build, A/B of
+# the prebuilt variants in ab_ship/, ncu pipe counters of selected variants.
+#   bash tools/r02_session.sh TAG "ab variants" "ncu variants" [steps...]
+TAG=$1; AB=$2; NCUV=$3; shift 3
+WHAT=${@:-tests bench ab ncu}
+mkdir -p gpurun_out
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/${TAG}_build.log 2>&1 || { echo build failed; exit 1; }
+for w in $WHAT; do
+case $w in
+tests)
+  timeout 1200 python -m pytest tests -m gpu -x -q > gpurun_out/${TAG}_gpu_tests.log 2>&1; tail -3 gpurun_out/${TAG}_gpu_tests.log
+  timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/${TAG}_smoke.log 2>&1; tail -1 gpurun_out/${TAG}_smoke.log ;;
+bench)
+  timeout 600 python bench.py > gpurun_out/${TAG}_bench.json 2> gpurun_out/${TAG}_bench.err; cat gpurun_out/${TAG}_bench.json ;;
+ab)
+  timeout 1200 python tools/ab_ship.py time 36 512 2 $AB > gpurun_out/${TAG}_ab.jsonl 2>&1
+  python tools/ab_summary.py gpurun_out/${TAG}_ab.jsonl ;;
+ncu)
+  for v in $NCUV; do
+    HPL_LIB=$PWD/ab_ship/libhpl_$v.so timeout 300 ncu --clock-control none -k regex:ep_kernel -s 1 -c 1 \
+      --metrics gpu__time_duration.sum,sm__pipe_fp64_cycles_active.avg.pct_of_peak_sustained_active,smsp__issue_active.avg.pct_of_peak_sustained_active,smsp__inst_executed.sum,sm__inst_executed_pipe_fp64.sum,smsp__inst_executed_pipe_fp64.sum,sm__cycles_elapsed.avg,smsp__average_warps_issue_stalled_dispatch_stall_per_issue_active.ratio,smsp__average_warps_issue_stalled_math_pipe_throttle_per_issue_active.ratio,smsp__average_warps_issue_stalled_not_selected_per_issue_active.ratio,smsp__average_warps_issue_stalled_wait_per_issue_active.ratio,smsp__average_warps_issue_stalled_short_scoreboard_per_issue_active.ratio \
+      --csv python tools/quick_time.py 32 --threads 512 --reps 1 > gpurun_out/${TAG}_ncu_$v.csv 2>&1
+  done ;;
+fc)
+  for v in ${FCV:-def}; do
+    HPL_LIB=$PWD/ab_ship/libhpl_$v.so timeout 300 python tools/fixed_cost.py ${FCM:-10,24,25,27} >> gpurun_out/${TAG}_fc.jsonl 2>&1
+  done
+  cat gpurun_out/${TAG}_fc.jsonl ;;
+ncufull)
+  timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${TAG}_launches.csv \
+      python bench.py --steps 2 --warmup 3 --no-cpu-baseline > gpurun_out/${TAG}_ncu_bench.log 2>&1
+  timeout 900 ncu --set full --clock-control none --import-source on -k regex:ep_kernel -s 3 -c 1 \
+      -o gpurun_out/${TAG}_prof -f python bench.py --steps 1 --warmup 3 --no-cpu-baseline > gpurun_out/${TAG}_ncu_full.log 2>&1
+  tail -2 gpurun_out/${TAG}_ncu_full.log ;;
+shard)
+  timeout 900 python tools/shard_timing.py > gpurun_out/${TAG}_shard.jsonl 2>&1; tail -4 gpurun_out/${TAG}_shard.jsonl ;;
+esac
+done
