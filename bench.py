@@ -46,7 +46,7 @@ ALG_OPS_ALWAYS = 6
 ALG_OPS_ACCEPTED = 18
 P_ACCEPT = 0.7853981633974483
 ALG_OPS_PER_PAIR = ALG_OPS_ALWAYS + P_ACCEPT * ALG_OPS_ACCEPTED
-EXEC_FP64_PER_PAIR = 22             # SASS of the hot loop (tools/sass_hot.py): DFMA 10 + DMUL 7 + DADD 5
+EXEC_FP64_PER_PAIR = 20             # SASS of the hot loop (tools/sass_hot.py): DFMA 10 + DMUL 6 + DADD 4
 FP64_LANES_PER_SM_CLK = 64          # measured: tools/probe_fp64.cu (63.9-64.1 lane-DFMA/clk/SM)
 EP_PARAM_BYTES = 560                 # EPParams kernel-parameter block (jump table, a^k table, coefs, scalars)
 

@@ -13,6 +13,8 @@ tests)
   timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/${TAG}_smoke.log 2>&1; tail -1 gpurun_out/${TAG}_smoke.log ;;
 bench)
   timeout 600 python bench.py > gpurun_out/${TAG}_bench.json 2> gpurun_out/${TAG}_bench.err; cat gpurun_out/${TAG}_bench.json ;;
+ref)
+  timeout 600 python bench.py --impl reference > gpurun_out/${TAG}_ref.json 2> gpurun_out/${TAG}_ref.err; cat gpurun_out/${TAG}_ref.json ;;
 ab)
   timeout 1200 python tools/ab_ship.py time 36 512 2 $AB > gpurun_out/${TAG}_ab.jsonl 2>&1
   python tools/ab_summary.py gpurun_out/${TAG}_ab.jsonl ;;
