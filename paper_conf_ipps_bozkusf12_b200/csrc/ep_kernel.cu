@@ -62,8 +62,13 @@ __device__ __forceinline__ double rsqrt_approx(double p) {
 
 // Shared-memory address of the log-table entry of t' (high word H).  `tabb` is
 // the table base, pre-biased by -TRUNC_J0 entries in the truncating mode.
-__device__ __forceinline__ unsigned tab_addr(unsigned H, unsigned tabb) {
-#if EP_IDX_TRUNC && EP_T_FMA == 2
+#ifndef EP_IDX_ONE
+#define EP_IDX_ONE 0  // 1: the +1 of the fused-t' index from a loop-invariant register (-0.33 IMAD.MOV/pair; measured -2.7 %)
+#endif
+__device__ __forceinline__ unsigned tab_addr(unsigned H, unsigned tabb, unsigned one = 1u) {
+#if EP_IDX_TRUNC && EP_T_FMA == 2 && EP_IDX_ONE
+  return ((max(H + one, TRUNC_HLO) >> LOG_SHIFT) << 4) + tabb;
+#elif EP_IDX_TRUNC && EP_T_FMA == 2
   // H + 1: the fused t' with high word 0x3FCFFFFF (just below 1/4) shares the
   // NaN bucket of [1/4, 1/4 + w) -> rare path (exact acceptance); other t'
   // move at most one high-word step (|r| <= 2^-10 + 2^-20)
@@ -495,7 +500,7 @@ struct Stage {
 
 template <bool A32, int W>
 __device__ __forceinline__ void gen_stage(unsigned& vlo, unsigned& vhi, const EPParams& P, unsigned tab,
-                                          Stage<W>& S, unsigned exp_hi) {
+                                          Stage<W>& S, unsigned exp_hi, unsigned one = 1u) {
 #pragma unroll
   for (int k = 0; k < W; ++k) {
 #if EP_ABL & 2  // ablation (timing only, wrong results): LCG step -> one add
@@ -551,7 +556,7 @@ __device__ __forceinline__ void gen_stage(unsigned& vlo, unsigned& vhi, const EP
     S.eInv[k] = S.x2[k];
 #elif EP_IDX_TRUNC
     asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(S.eT[k]), "=d"(S.eInv[k])
-                 : "r"(tab_addr(static_cast<unsigned>(__double2hiint(S.t[k])), tab)));
+                 : "r"(tab_addr(static_cast<unsigned>(__double2hiint(S.t[k])), tab, one)));
 #else
     asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(S.eT[k]), "=d"(S.eInv[k]) : "r"((S.u[k] << 4) + tab));
 #endif
@@ -828,7 +833,7 @@ __device__ EP_LOOP_INL LoopOut pair_loop(unsigned vlo, unsigned vhi, uint64_t n_
     uint64_t iters = P.base / PER_IT;
     const LeanConst K = make_lean_const(kc);
     Stage<W> s0, s1;
-    gen_stage<A32, W>(vlo, vhi, P, tab, s0, K.exp_hi);
+    gen_stage<A32, W>(vlo, vhi, P, tab, s0, K.exp_hi, K.one);
     while (iters) {
       const unsigned ci = iters < IT_PER_CHUNK ? unsigned(iters) : IT_PER_CHUNK;
       PairAcc A{0.0, 0.0, 0u};
@@ -836,12 +841,12 @@ __device__ EP_LOOP_INL LoopOut pair_loop(unsigned vlo, unsigned vhi, uint64_t n_
       for (unsigned i = 0; i < ci; ++i) {
 #if EP_PIPE_ORDER == 1
         transform_stage<W>(s0, P, K, A, s_rare);
-        gen_stage<A32, W>(vlo, vhi, P, tab, s0, K.exp_hi);
+        gen_stage<A32, W>(vlo, vhi, P, tab, s0, K.exp_hi, K.one);
         (void)s1;
 #else
-        gen_stage<A32, W>(vlo, vhi, P, tab, s1, K.exp_hi);
+        gen_stage<A32, W>(vlo, vhi, P, tab, s1, K.exp_hi, K.one);
         transform_stage<W>(s0, P, K, A, s_rare);
-        gen_stage<A32, W>(vlo, vhi, P, tab, s0, K.exp_hi);
+        gen_stage<A32, W>(vlo, vhi, P, tab, s0, K.exp_hi, K.one);
         transform_stage<W>(s1, P, K, A, s_rare);
 #endif
       }
@@ -853,7 +858,7 @@ __device__ EP_LOOP_INL LoopOut pair_loop(unsigned vlo, unsigned vhi, uint64_t n_
       PairAcc A{0.0, 0.0, 0u};
       transform_stage<W>(s0, P, K, A, s_rare, nullptr, tail < W ? tail : W);
 #if EP_PIPE_ORDER != 1
-      gen_stage<A32, W>(vlo, vhi, P, tab, s1, K.exp_hi);
+      gen_stage<A32, W>(vlo, vhi, P, tab, s1, K.exp_hi, K.one);
       transform_stage<W>(s1, P, K, A, s_rare, nullptr, tail > W ? tail - W : 0u);
 #endif
       flush(A);

@@ -22,7 +22,7 @@ if sys.argv[1] == "build":
         x = tuple(y for x in items if x.startswith("-") for y in x.split())
         build.build(out=os.path.join(OUT, "libhpl_%s.so" % name), defines=d, extra=x)
         return name, d, x
-    with ThreadPoolExecutor(max_workers=4) as ex:
+    with ThreadPoolExecutor(max_workers=int(os.environ.get("AB_J", "4"))) as ex:
         for r in ex.map(one, sys.argv[2:]):
             print("built", *r, flush=True)
 else:

@@ -13,6 +13,8 @@ tests)
   timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/${TAG}_smoke.log 2>&1; tail -1 gpurun_out/${TAG}_smoke.log ;;
 bench)
   timeout 600 python bench.py > gpurun_out/${TAG}_bench.json 2> gpurun_out/${TAG}_bench.err; cat gpurun_out/${TAG}_bench.json ;;
+ptest)
+  HPL_LIB=$PWD/ab_ship/libhpl_${PTV}.so timeout 1200 python -m pytest tests/test_gpu_parity.py tests/test_edge_pairs.py tests/test_fused_combine.py tests/test_gpu_accuracy.py -m gpu -x -q > gpurun_out/${TAG}_ptest_${PTV}.log 2>&1; tail -3 gpurun_out/${TAG}_ptest_${PTV}.log ;;
 ref)
   timeout 600 python bench.py --impl reference > gpurun_out/${TAG}_ref.json 2> gpurun_out/${TAG}_ref.err; cat gpurun_out/${TAG}_ref.json ;;
 ab)
