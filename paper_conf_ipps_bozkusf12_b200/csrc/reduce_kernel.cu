@@ -71,13 +71,16 @@ reduce_sum_f32_kernel(const float* __restrict__ in, int64_t n, double* __restric
     for (unsigned w = 0; w < blockDim.x / 32; ++w) b += s_w[w];
     partials[blockIdx.x] = b;
     __threadfence();
-    s_last = atomicAdd(counter, 1u) == gridDim.x - 1;
+    // acquiring ticket: the last block's loads below (after the barrier) are
+    // ordered after every block's fence + ticket (no second fence)
+    unsigned ticket;
+    asm volatile("atom.add.acquire.gpu.global.u32 %0, [%1], 1;" : "=r"(ticket) : "l"(counter) : "memory");
+    s_last = ticket == gridDim.x - 1;
   }
   __syncthreads();
   if (!s_last) return;
   // last block: all threads fold the partials (strided, fixed order), then
   // the same warp/block tree — deterministic, and no serial 600-load chain
-  __threadfence();
   double s = 0.0;
   for (unsigned b = threadIdx.x; b < gridDim.x; b += blockDim.x) s += __ldcg(partials + b);
 #pragma unroll
