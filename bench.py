@@ -293,7 +293,25 @@ def run_ours(args, M):
             dist.all_reduce(out)
     torch.cuda.synchronize(dev)
     if combine == "fused":
-        fc.status()  # raises if a warm-up combine timed out
+        # the first multi-GPU execution of the peer-memory combine is here: if a
+        # warm-up call timed out, tore a slot or produced a result that fails
+        # verification on any rank, every rank switches to the NCCL combine
+        # (agreed over NCCL, which does not depend on the fused path)
+        try:
+            fc.status()
+            ok = verify_result(args.cls, M, hpl.unpack13(out.cpu().tolist()), world)["ok"]
+            why = "warm-up result failed verification"
+        except hpl.HPLError as e:
+            ok, why = False, "warm-up combine failed: %s" % str(e)[:160]
+        flag = torch.tensor([1.0 if ok else 0.0], device=dev)
+        dist.all_reduce(flag, op=dist.ReduceOp.MIN)
+        if flag.item() == 0.0:
+            combine = "nccl"
+            combine_note = why if not ok else "fused combine failed on a peer rank"
+            for _ in range(max(args.warmup, 1)):
+                step()
+                dist.all_reduce(out)
+            torch.cuda.synchronize(dev)
 
     # ---- device-timed region
     sampler = ClockSampler(gpu)

@@ -1,12 +1,18 @@
 """Generic eval over index domains: the paper's own example
-kernels run through hpl_eval, checked against their plain definitions
-(numpy, IEEE roundings as the kernels write them) and the paper's Fig. 2
-statement about local ids.
+kernels run through hpl_eval, checked against oracle/eval_f1.py (plain
+definitions of Figs. 2-4 in the paper's order and roundings) and the paper's
+Fig. 2 statement about local ids.  The oracle itself is pinned here on CPU:
+Fig. 2's printed ids, exact rational arithmetic with correct rounding for
+saxpy and for dotp's float32 chain.
 """
 import ctypes
+import random
+from fractions import Fraction
 
 import numpy as np
 import pytest
+
+from oracle import eval_f1
 
 
 @pytest.fixture(scope="module")
@@ -30,6 +36,63 @@ def test_bad_calls_rejected_without_gpu(hpl):
         with pytest.raises(hpl.HPLError) as e:
             hpl.hpl_eval(name, args)
         assert e.value.code == hpl.HPL_EINVAL
+
+
+# ------------------------------------------------------- oracle pins (CPU)
+def _rn32(fr: Fraction) -> np.float32:
+    """Correctly rounded float32 of an exact rational (ties to even)."""
+    f = np.float32(float(fr))
+    cands = [f, np.nextafter(f, np.float32(np.inf)), np.nextafter(f, np.float32(-np.inf))]
+    best = min(cands, key=lambda c: (abs(Fraction(float(c)) - fr), int(np.float32(c).view(np.int32)) & 1))
+    return np.float32(best)
+
+
+def test_oracle_fig2_ids_as_printed():
+    """global 4x8, local 2x4 — the points (1,2), (1,6), (3,2)
+    and (3,6) all have local id (1,2); ids partition the domain."""
+    ids = eval_f1.domain_ids([4, 8], [2, 4])
+    assert ids.shape == (32, 9)
+    for (x, y) in [(1, 2), (1, 6), (3, 2), (3, 6)]:
+        assert tuple(ids[y * 4 + x, 3:5]) == (1, 2)
+    assert np.array_equal(ids[:, 0:3], ids[:, 6:9] * np.array([2, 4, 1]) + ids[:, 3:6])
+    assert len({tuple(r[0:3]) for r in ids}) == 32
+    assert set(map(tuple, ids[:, 6:8])) == {(gx, gy) for gx in range(2) for gy in range(2)}
+
+
+def test_oracle_saxpy_two_roundings():
+    """y = RN(RN(a x) + y) by exact rationals + correct rounding (float()),
+    including inputs where an fma would give a different double."""
+    rng = random.Random(5)
+    xs = [rng.uniform(-1e3, 1e3) for _ in range(500)] + [1.0 + 2.0 ** -30]
+    ys = [rng.uniform(-1e3, 1e3) for _ in range(500)] + [-(1.0 + 2.0 ** -29)]
+    a = 1.0 + 2.0 ** -30
+    got = eval_f1.saxpy(ys, xs, a)
+    for g, x, y in zip(got, xs, ys):
+        want = float(Fraction(float(Fraction(a) * Fraction(x))) + Fraction(y))
+        assert float(g) == want
+    # the constructed last element: an fma keeps a*x's low bits, two roundings lose them
+    fused = float(Fraction(a) * Fraction(xs[-1]) + Fraction(ys[-1]))
+    assert float(got[-1]) != fused
+
+
+@pytest.mark.parametrize("M", [1, 4, 32])
+def test_oracle_dotp_float32_chain(M):
+    """Fig. 4: each partial is lane 0's in-order float32 sum of float32
+    products — checked against exact rationals rounded to float32 at every
+    step, and against a float64 dot product."""
+    rng = np.random.default_rng(M)
+    N = 8 * M
+    v1 = rng.standard_normal(N).astype(np.float32)
+    v2 = rng.standard_normal(N).astype(np.float32)
+    got = eval_f1.dotp(v1, v2, M)
+    for g in range(N // M):
+        acc = np.float32(0.0)
+        for i in range(M):
+            prod = _rn32(Fraction(float(v1[g * M + i])) * Fraction(float(v2[g * M + i])))
+            acc = _rn32(Fraction(float(acc)) + Fraction(float(prod)))
+        assert got[g] == acc
+    assert abs(float(got.astype(np.float64).sum()) - float(np.dot(v1.astype(np.float64), v2.astype(np.float64)))) \
+        < 1e-5 * N
 
 
 # ------------------------------------------------------------------- GPU
@@ -58,12 +121,7 @@ def test_fig2_domain_ids(gpu):
         hpl.hpl_eval("domain_ids", [a], global_=[gx, gy], local=[lx, ly])
         hpl.hpl_array_sync(a, hpl.HPL_HOST, hpl.HPL_READ)
         ids = _host(hpl, a, np.int32, gx * gy * 9).reshape(gy, gx, 9)
-        for y in range(gy):
-            for x in range(gx):
-                i = ids[y, x]
-                assert tuple(i[0:3]) == (x, y, 0)
-                assert tuple(i[3:6]) == (x % lx, y % ly, 0)
-                assert tuple(i[6:9]) == (x // lx, y // ly, 0)
+        assert np.array_equal(ids.reshape(-1, 9), eval_f1.domain_ids([gx, gy], [lx, ly]))
         for (x, y) in [(1, 2), (1, 6), (3, 2), (3, 6)]:
             assert tuple(ids[y, x, 3:5]) == (1, 2)
     finally:
@@ -112,14 +170,14 @@ def test_fig3_saxpy(gpu):
         assert hpl.hpl_array_info(y)["valid"] == hpl.HPL_DEVICE
         assert np.array_equal(myvector, y0)  # host copy untouched until synced
         hpl.hpl_array_sync(y, hpl.HPL_HOST, hpl.HPL_READ)
-        assert np.array_equal(myvector, a * xh + y0)
+        assert np.array_equal(myvector, eval_f1.saxpy(y0, xh, a))
         # a second eval reuses the still-valid device copy of x: a host edit
         # not announced with a WRITE sync is (by contract) not uploaded
         x_old, y1 = xh.copy(), myvector.copy()
         xh[:] = 0.0
         hpl.hpl_eval("saxpy", [y, x, a])
         hpl.hpl_array_sync(y, hpl.HPL_HOST, hpl.HPL_READ)
-        assert np.array_equal(myvector, a * x_old + y1)
+        assert np.array_equal(myvector, eval_f1.saxpy(y1, x_old, a))
         # announcing the edit makes the next eval upload it
         hpl.hpl_array_sync(x, hpl.HPL_HOST, hpl.HPL_WRITE)
         y2 = myvector.copy()
@@ -151,11 +209,7 @@ def test_fig4_dotp(gpu, N, M):
             hpl.hpl_array_sync(h, hpl.HPL_HOST, hpl.HPL_WRITE)
         hpl.hpl_eval("dotp", [v1, v2, ps], global_=[N], local=[M])
         hpl.hpl_array_sync(ps, hpl.HPL_HOST, hpl.HPL_READ)
-        prods = (a1 * a2).astype(np.float32).reshape(ng, M)
-        want = np.zeros(ng, dtype=np.float32)
-        for i in range(M):  # lane 0's sequential float32 sum
-            want = (want + prods[:, i]).astype(np.float32)
-        assert np.array_equal(p, want)
+        assert np.array_equal(p, eval_f1.dotp(a1, a2, M))
         dot = float(np.sum(p.astype(np.float64)))
         assert abs(dot - float(np.dot(a1.astype(np.float64), a2.astype(np.float64)))) < 1e-3 * N ** 0.5
     finally:

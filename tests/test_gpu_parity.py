@@ -129,8 +129,6 @@ def test_npb_large_class_vs_golden(env, variant, cls):
     gold = oracle_golden().get(cls)
     if gold is None:
         pytest.skip("tests/golden/oracle_ep.json lacks class %s" % cls)
-    if variant == 1 and cls == "D":
-        pytest.skip("libdevice variant at class D is covered by bench A/B runs")
     hpl.hpl_ep_set_config(variant, 0, 0)
     sx, sy, q = hpl.hpl_ep_run(gold["M"], NPB_SEED, NPB_A)
     hpl.hpl_ep_set_config(0, 0, 0)
