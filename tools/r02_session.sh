@@ -17,6 +17,8 @@ ptest)
   HPL_LIB=$PWD/ab_ship/libhpl_${PTV}.so timeout 1200 python -m pytest tests/test_gpu_parity.py tests/test_edge_pairs.py tests/test_fused_combine.py tests/test_gpu_accuracy.py -m gpu -x -q > gpurun_out/${TAG}_ptest_${PTV}.log 2>&1; tail -3 gpurun_out/${TAG}_ptest_${PTV}.log ;;
 gloo2)
   bash tools/bench_gloo2.sh > gpurun_out/${TAG}_gloo2.log 2>&1; cp gpurun_out/b2_fused.json gpurun_out/${TAG}_b2_fused.json; cp gpurun_out/b2_nccl.json gpurun_out/${TAG}_b2_nccl.json; tail -8 gpurun_out/${TAG}_gloo2.log ;;
+san)
+  bash tools/sanitize.sh > gpurun_out/${TAG}_sanitize.log 2>&1; for t in memcheck racecheck synccheck; do cp gpurun_out/sanitize_$t.log gpurun_out/${TAG}_sanitize_$t.log; done; cat gpurun_out/${TAG}_sanitize.log ;;
 ref)
   timeout 600 python bench.py --impl reference > gpurun_out/${TAG}_ref.json 2> gpurun_out/${TAG}_ref.err; cat gpurun_out/${TAG}_ref.json ;;
 ab)
