@@ -193,10 +193,12 @@ __device__ __forceinline__ void lcg_step(unsigned& lo, unsigned& hi, unsigned a_
 }
 
 
-// -2 ln(1+r) = r (-2 + r (1 + r (-2/3 + r (1/2 + r (c5 + r c6))))), |r| <= 2^-9.
-// c5 = -2/5 and c6 = 1/3 only weigh r^5, r^6 terms (< 2^-36 relative), so they
-// are rounded to 20-bit mantissas that encode as DFMA immediates (relative
-// effect < 2^-60); -2/3 stays exact (kernel parameter).  DESIGN.md §4.2.
+// -2 ln(1+r) = r (-2 + r (1 + r (-2/3 + r (1/2 + r (c5 + r c6))))).  The default
+// (EP_LOG_DEG4, K = 9 table, |r| <= 2^-10) stops at r/2: the dropped (2/5) r^5
+// is <= (2/5) 2^-50 in L (R11).  The longer series of the other
+// modes (K = 8, or EP_LOG_DEG4=0) rounds c5 = -2/5 and c6 = 1/3 to 20-bit
+// mantissas that encode as DFMA immediates (they only weigh r^5, r^6: relative
+// effect < 2^-60); -2/3 stays exact (kernel parameter).
 #define EP_C6 0x1.55555p-2    /* 1/3  rounded to 20 bits */
 #define EP_C5 -0x1.9999ap-2   /* -2/5 rounded to 20 bits */
 
@@ -1268,7 +1270,7 @@ static EPKernel tier_kernel(int thr) {
 #define EP_T384_W EP_ILP
 #endif
 #ifndef EP_T512_W
-#define EP_T512_W 3  // 124 registers, no spills; +2 % over W = 2
+#define EP_T512_W 3  // 120 registers, no spills (round 2: W = 2 is 4 % slower, W = 4 spills)
 #endif
   if (thr <= 128) return ep_kernel<V, A32, 128, 4, 1>;   // 128 regs
   if (thr <= 256) return ep_kernel<V, A32, 256, EP_T256_MINB, EP_T256_W>;   //  85 regs (3 blocks/SM)
