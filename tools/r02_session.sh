@@ -19,6 +19,11 @@ gloo2)
   bash tools/bench_gloo2.sh > gpurun_out/${TAG}_gloo2.log 2>&1; cp gpurun_out/b2_fused.json gpurun_out/${TAG}_b2_fused.json; cp gpurun_out/b2_nccl.json gpurun_out/${TAG}_b2_nccl.json; tail -8 gpurun_out/${TAG}_gloo2.log ;;
 san)
   bash tools/sanitize.sh > gpurun_out/${TAG}_sanitize.log 2>&1; for t in memcheck racecheck synccheck; do cp gpurun_out/sanitize_$t.log gpurun_out/${TAG}_sanitize_$t.log; done; cat gpurun_out/${TAG}_sanitize.log ;;
+evalb)
+  timeout 600 python -m pytest tests/test_eval.py -m gpu -q > gpurun_out/${TAG}_evaltests.log 2>&1; tail -2 gpurun_out/${TAG}_evaltests.log
+  timeout 600 python tools/bench_eval.py > gpurun_out/${TAG}_eval.jsonl 2>&1
+  HPL_LIB=$PWD/ab_ship/libhpl_nopipe.so timeout 600 python tools/bench_eval.py > gpurun_out/${TAG}_eval_nopipe.jsonl 2>&1
+  cat gpurun_out/${TAG}_eval.jsonl gpurun_out/${TAG}_eval_nopipe.jsonl ;;
 ref)
   timeout 600 python bench.py --impl reference > gpurun_out/${TAG}_ref.json 2> gpurun_out/${TAG}_ref.err; cat gpurun_out/${TAG}_ref.json ;;
 ab)
