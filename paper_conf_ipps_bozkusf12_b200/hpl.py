@@ -48,7 +48,12 @@ HPL_ARG_ARRAY, HPL_ARG_F64, HPL_ARG_F32, HPL_ARG_I64, HPL_ARG_I32 = 0, 1, 2, 3, 
 # hpl_alloc_fn / hpl_free_fn (include/hpl.h)
 _ALLOC_T = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_int, ctypes.c_void_p)
 _FREE_T = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_size_t, ctypes.c_int, ctypes.c_void_p)
-_allocator = None  # the installed callbacks (kept alive here)
+_allocator = None  # the installed callbacks
+# every callback pair ever installed stays referenced for the life of the
+# process: arrays remember the allocator that made them, and one allocated
+# under callbacks that were later replaced (or by another thread whose
+# per-thread cache outlives hpl_shutdown) still frees through them
+_keepalive = []
 
 
 class HplArg(ctypes.Structure):
@@ -151,6 +156,7 @@ def hpl_set_device_allocator(alloc=None, free=None) -> None:
         return
     cb = (_ALLOC_T(lambda n, dev, ctx: alloc(n, dev) or None),
           _FREE_T(lambda p, n, dev, ctx: free(p, n, dev)))
+    _keepalive.append(cb)
     _check(lib.hpl_set_device_allocator(cb[0], cb[1], None), "hpl_set_device_allocator")
     _allocator = cb
 
