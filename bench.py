@@ -46,6 +46,9 @@ ALG_OPS_ALWAYS = 6
 ALG_OPS_ACCEPTED = 18
 P_ACCEPT = 0.7853981633974483
 ALG_OPS_PER_PAIR = ALG_OPS_ALWAYS + P_ACCEPT * ALG_OPS_ACCEPTED
+# algorithmic-fraction ceiling of the minimal instruction mix (DESIGN.md §5,
+# profiles/r02_ceiling.md): 2 / (1.93 + 1.03 * 0.72) of the FP64 pipe x 20.137 / 20
+CEILING_FRAC = 0.754
 EXEC_FP64_PER_PAIR = 20             # SASS of the hot loop (tools/sass_hot.py): DFMA 10 + DMUL 6 + DADD 4
 FP64_LANES_PER_SM_CLK = 64          # measured: tools/probe_fp64.cu (63.9-64.1 lane-DFMA/clk/SM)
 EP_PARAM_BYTES = 560                 # EPParams kernel-parameter block (jump table, a^k table, coefs, scalars)
@@ -438,7 +441,11 @@ def run_ours(args, M):
                          # executes per pair (every pair runs the transform) / peak
                          "executed_fp64_per_pair": EXEC_FP64_PER_PAIR,
                          "fp64_pipe_frac": round(achieved / peak_ops * EXEC_FP64_PER_PAIR / ALG_OPS_PER_PAIR, 4),
-                         "ncu_fp64_pipe_active_pct": load_profile_field("fp64_pipe_active_pct")},
+                         "ncu_fp64_pipe_active_pct": load_profile_field("fp64_pipe_active_pct"),
+                         # counter-backed ceiling of this instruction mix (profiles/r02_ceiling.md):
+                         # cycles/FP64 instr = 1.93 + 1.03 rho, rho >= 0.72 non-FP64 instr per FP64
+                         "instruction_mix_ceiling_frac": CEILING_FRAC,
+                         "frac_of_ceiling": round(achieved / peak_ops / CEILING_FRAC, 4)},
             "e2e": {"value": round(units * args.steps / (e2e_tot / 1e3) / 1e6, 1), "unit": UNIT,
                     "h2d_bytes_per_step": EP_PARAM_BYTES * world, "d2h_bytes_per_step": 104 * world,
                     "note": "h2d = kernel-parameter block (jump table + scalars); d2h = 13-word result"},

@@ -478,6 +478,9 @@ constexpr int kLoopUnroll = EP_LOOP_UNROLL;  // (#pragma arguments are not macro
 #if EP_PRED_MODE == 1 && EP_BIN_MODE != 3
 #error "EP_PRED_MODE 1 needs EP_BIN_MODE 3"
 #endif
+#if EP_PRED_MODE == 1 && EP_T_FMA
+#error "EP_PRED_MODE 1 reads acceptance from the selector, which cannot tell the fused t' next to 1/4 (EP_T_FMA) from a reject"
+#endif
 #ifndef EP_RARE_VOTE
 #define EP_RARE_VOTE 1 // 1: rare-path branch on a warp vote (needs warp-uniform trip counts)
 #endif
@@ -688,7 +691,7 @@ __device__ __forceinline__ void transform_stage(const Stage<W>& S, const EPParam
     // selector bits: < 2^20 + 4/8 ok; [.., 2^21) rare (l >= 4 or tiny t');
     // >= 2^21 or NaN: rejected (reject sentinel, or t' > 1/4 in the 1/4 bucket,
     // where L < 0 makes X, Y NaN and FMNMX3.NAN propagates it)
-    sel_min = min(sel_min, l[k] - 0x49800004u);
+    if (k < nvalid) sel_min = min(sel_min, l[k] - 0x49800004u);  // (masked tail pairs never reach the rare path)
 #endif
     if (ok[k]) {
 #if EP_MAXSQ
@@ -726,7 +729,7 @@ __device__ __forceinline__ void transform_stage(const Stage<W>& S, const EPParam
 #endif
 #pragma unroll
     for (int k = 0; k < W; ++k)
-      if (EP_PRED_MODE == 1 ? (l[k] - 0x49800004u < 0x007FFFFCu) : ((acc[k] && !ok[k]) || band[k])) {
+      if (EP_PRED_MODE == 1 ? (k < nvalid && l[k] - 0x49800004u < 0x007FFFFCu) : ((acc[k] && !ok[k]) || band[k])) {
         if (EP_MAXSQ) {
           X[k] = __dmul_rn(S.x1[k], t2[k]);
           Y[k] = __dmul_rn(S.x2[k], t2[k]);
