@@ -24,6 +24,11 @@ evalb)
   timeout 600 python tools/bench_eval.py > gpurun_out/${TAG}_eval.jsonl 2>&1
   HPL_LIB=$PWD/ab_ship/libhpl_nopipe.so timeout 600 python tools/bench_eval.py > gpurun_out/${TAG}_eval_nopipe.jsonl 2>&1
   cat gpurun_out/${TAG}_eval.jsonl gpurun_out/${TAG}_eval_nopipe.jsonl ;;
+redb)
+  HPL_LIB=$PWD/ab_ship/libhpl_rtma.so timeout 600 python -m pytest tests/test_reduce.py -m gpu -q > gpurun_out/${TAG}_redtests.log 2>&1; tail -2 gpurun_out/${TAG}_redtests.log
+  for v in ${REDV:-ship rtma}; do echo "== $v" >> gpurun_out/${TAG}_red.jsonl; HPL_LIB=$PWD/ab_ship/libhpl_$v.so timeout 300 python tools/bench_reduce.py --n 16777216 268435456 >> gpurun_out/${TAG}_red.jsonl 2>&1; done
+  for v in ${REDV:-ship rtma}; do HPL_LIB=$PWD/ab_ship/libhpl_$v.so timeout 300 ncu --clock-control none -k regex:reduce_sum --metrics gpu__time_duration.sum,dram__bytes_read.sum --csv python tools/bench_reduce.py --n 16777216 --iters 3 > gpurun_out/${TAG}_red_ncu_$v.csv 2>&1; done
+  cat gpurun_out/${TAG}_red.jsonl ;;
 ref)
   timeout 600 python bench.py --impl reference > gpurun_out/${TAG}_ref.json 2> gpurun_out/${TAG}_ref.err; cat gpurun_out/${TAG}_ref.json ;;
 ab)
