@@ -29,6 +29,8 @@ redb)
   for v in ${REDV:-ship rtma}; do echo "== $v" >> gpurun_out/${TAG}_red.jsonl; HPL_LIB=$PWD/ab_ship/libhpl_$v.so timeout 300 python tools/bench_reduce.py --n 16777216 268435456 >> gpurun_out/${TAG}_red.jsonl 2>&1; done
   for v in ${REDV:-ship rtma}; do HPL_LIB=$PWD/ab_ship/libhpl_$v.so timeout 300 ncu --clock-control none -k regex:reduce_sum --metrics gpu__time_duration.sum,dram__bytes_read.sum --csv python tools/bench_reduce.py --n 16777216 --iters 3 > gpurun_out/${TAG}_red_ncu_$v.csv 2>&1; done
   cat gpurun_out/${TAG}_red.jsonl ;;
+classes)
+  for c in S W A B C; do timeout 300 python bench.py --cls $c --steps 20 --warmup 5 --no-cpu-baseline > gpurun_out/${TAG}_bench_$c.json 2>/dev/null; python -c "import json;d=json.load(open('gpurun_out/${TAG}_bench_$c.json'));print('$c', d['value'], d['ms_per_step'], d['verified'], d['roofline']['frac'])"; done ;;
 ref)
   timeout 600 python bench.py --impl reference > gpurun_out/${TAG}_ref.json 2> gpurun_out/${TAG}_ref.err; cat gpurun_out/${TAG}_ref.json ;;
 ab)
