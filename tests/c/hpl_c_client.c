@@ -3,7 +3,9 @@
  *   gpu  : NPB class S through hpl_ep_run and the Array/eval path, checked
  *          against NPB's published verification sums (tests/golden); the
  *          transpose through eval on Arrays and the reduction on an Array's
- *          device copy, checked against their definitions */
+ *          device copy, checked against their definitions; a caller-installed
+ *          device allocator (counting, over cudart) and hpl_shutdown */
+#include <cuda_runtime_api.h>
 #include <math.h>
 #include <stdio.h>
 #include <string.h>
@@ -12,6 +14,24 @@
 
 static int fails = 0;
 #define CHECK(c) do { if (!(c)) { printf("FAIL %s:%d %s\n", __FILE__, __LINE__, #c); ++fails; } } while (0)
+
+/* counting allocator over the CUDA runtime (caller-side, for the test) */
+static int g_allocs = 0, g_frees = 0, g_ctx_tag = 0;
+static size_t g_alloc_bytes = 0;
+static void* g_ctx_seen = NULL;
+static void* counting_alloc(size_t bytes, int device, void* ctx) {
+  void* p = NULL;
+  (void)device;
+  ++g_allocs;
+  g_alloc_bytes = bytes;
+  g_ctx_seen = ctx;
+  return cudaMalloc(&p, bytes) == cudaSuccess ? p : NULL;
+}
+static void counting_free(void* p, size_t bytes, int device, void* ctx) {
+  (void)bytes; (void)device; (void)ctx;
+  ++g_frees;
+  cudaFree(p);
+}
 
 int main(int argc, char** argv) {
   const int gpu = argc > 1 && strcmp(argv[1], "gpu") == 0;
@@ -89,6 +109,23 @@ int main(int argc, char** argv) {
     const double n = (double)(H * W), want = 0.5 * n * (n - 1) / 2.0 - 100.0 * n;
     CHECK(*hsum == want);
     CHECK(hpl_array_free(src) == HPL_OK && hpl_array_free(dst) == HPL_OK && hpl_array_free(sum) == HPL_OK);
+
+    /* a caller-installed device allocator (include/hpl.h): Arrays draw from it
+       and return to it; after hpl_shutdown the library re-creates its state */
+    CHECK(hpl_set_device_allocator(counting_alloc, counting_free, &g_ctx_tag) == HPL_OK);
+    hpl_array c13;
+    CHECK(hpl_array_alloc(&c13, HPL_F64, 1, &d, NULL, -1) == HPL_OK);
+    CHECK(g_allocs == 1 && g_alloc_bytes == 104 && g_ctx_seen == &g_ctx_tag);
+    CHECK(hpl_ep_eval(20, 271828183ull, 1220703125ull, 0, 1, c13) == HPL_OK);
+    CHECK(hpl_array_sync(c13, HPL_HOST, HPL_READ) == HPL_OK);
+    CHECK(hpl_array_free(c13) == HPL_OK);
+    CHECK(g_frees == 1);
+    CHECK(hpl_shutdown() == HPL_OK);  /* frees the library's own buffers, resets the allocator */
+    CHECK(hpl_ep_run(20, 271828183ull, 1220703125ull, &sx, &sy, q) == HPL_OK);
+    CHECK(g_allocs == 1);             /* cudaMalloc again after hpl_shutdown */
+    gc = 0;
+    for (int i = 0; i < 10; ++i) gc += q[i];
+    CHECK(gc == 823561ull);           /* M = 20 (smoke value) */
   }
   printf("%s: %d failures\n", gpu ? "gpu" : "cpu", fails);
   return fails != 0;

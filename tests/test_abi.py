@@ -89,3 +89,12 @@ def test_null_outputs_rejected(hpl):
 
 def test_launch_counter_readable(hpl):
     assert hpl.hpl_ep_launch_count() >= 0
+
+
+def test_allocator_hook_validation(hpl):
+    """hpl_set_device_allocator: both callbacks or neither (include/hpl.h)."""
+    lib = hpl.lib()
+    alloc = hpl._ALLOC_T(lambda n, dev, ctx: None)
+    assert lib.hpl_set_device_allocator(alloc, hpl._FREE_T(), None) == hpl.HPL_EINVAL
+    assert lib.hpl_set_device_allocator(hpl._ALLOC_T(), hpl._FREE_T(lambda p, n, dev, ctx: None), None) == hpl.HPL_EINVAL
+    assert b"both" in hpl.lib().hpl_last_error()

@@ -13,9 +13,12 @@ def client(tmp_path_factory):
     from paper_conf_ipps_bozkusf12_b200 import build
     build.build()
     exe = str(tmp_path_factory.mktemp("c") / "hpl_c_client")
+    cuda = os.environ.get("CUDA_HOME", "/usr/local/cuda")  # the test's own allocator uses cudart
     subprocess.check_call(["gcc", "-O1", "-std=c99", "-Wall", "-I", os.path.join(ROOT, "include"),
+                           "-I", os.path.join(cuda, "include"),
                            os.path.join(ROOT, "tests", "c", "hpl_c_client.c"), "-L", PKG, "-lhpl",
-                           "-Wl,-rpath," + PKG, "-lm", "-o", exe])
+                           "-Wl,-rpath," + PKG, "-L", os.path.join(cuda, "lib64"), "-lcudart",
+                           "-Wl,-rpath," + os.path.join(cuda, "lib64"), "-lm", "-o", exe])
     return exe
 
 
