@@ -347,3 +347,16 @@ def test_acceptance_boundary_pairs(env, oracle_mod):
         begin = max(int(i) - (1 << 20), 0)
         g = gpu_range(env, NPB_SEED, NPB_A, begin, 1 << 21)
         assert_parity(g, oracle_mod.run_pairs(NPB_SEED, NPB_A, begin, 1 << 21))
+
+
+def test_arrays_draw_from_torchs_allocator(env):
+    """SURVEY §8(b) memory ownership: with torch loaded, hpl_array device
+    memory comes from torch's caching allocator (the binding installs it)."""
+    torch, hpl = env
+    before = torch.cuda.memory_allocated()
+    a = hpl.hpl_array_alloc(hpl.HPL_F64, [1 << 20])
+    try:
+        assert torch.cuda.memory_allocated() - before >= 8 << 20
+    finally:
+        hpl.hpl_array_free(a)
+    assert torch.cuda.memory_allocated() == before
