@@ -31,6 +31,10 @@ redb)
   cat gpurun_out/${TAG}_red.jsonl ;;
 classes)
   for c in S W A B C; do timeout 300 python bench.py --cls $c --steps 20 --warmup 5 --no-cpu-baseline > gpurun_out/${TAG}_bench_$c.json 2>/dev/null; python -c "import json;d=json.load(open('gpurun_out/${TAG}_bench_$c.json'));print('$c', d['value'], d['ms_per_step'], d['verified'], d['roofline']['frac'])"; done ;;
+evalab)
+  for v in ${EVV}; do echo "== $v" >> gpurun_out/${TAG}_evalab.jsonl; HPL_LIB=$PWD/ab_ship/libhpl_$v.so timeout 300 python tools/bench_eval.py >> gpurun_out/${TAG}_evalab.jsonl 2>&1; done
+  HPL_LIB=$PWD/ab_ship/libhpl_${PTV}.so timeout 600 python -m pytest tests/test_eval.py -m gpu -q > gpurun_out/${TAG}_evaltests.log 2>&1; tail -2 gpurun_out/${TAG}_evaltests.log
+  grep -v saxpy gpurun_out/${TAG}_evalab.jsonl | cut -c1-160 ;;
 ref)
   timeout 600 python bench.py --impl reference > gpurun_out/${TAG}_ref.json 2> gpurun_out/${TAG}_ref.err; cat gpurun_out/${TAG}_ref.json ;;
 ab)
