@@ -232,3 +232,28 @@ def test_eval_domain_errors(gpu):
     finally:
         hpl.hpl_array_free(a)
         hpl.hpl_array_free(b)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("dims", [[1], [7], [1001], [33, 31], [(1 << 20) + 3]])
+def test_saxpy_sizes(gpu, dims):
+    """Any domain size / rank: y = RN(RN(a x) + y) element by element (the
+    library may run several consecutive points per CUDA thread)."""
+    hpl = gpu
+    n = int(np.prod(dims))
+    rng = np.random.default_rng(n)
+    x = hpl.hpl_array_alloc(hpl.HPL_F64, dims)
+    y = hpl.hpl_array_alloc(hpl.HPL_F64, dims)
+    try:
+        xh, yh = _host(hpl, x, np.float64, n), _host(hpl, y, np.float64, n)
+        xh[:] = rng.standard_normal(n)
+        yh[:] = rng.standard_normal(n)
+        y0 = yh.copy()
+        for h in (x, y):
+            hpl.hpl_array_sync(h, hpl.HPL_HOST, hpl.HPL_WRITE)
+        hpl.hpl_eval("saxpy", [y, x, -0.75])
+        hpl.hpl_array_sync(y, hpl.HPL_HOST, hpl.HPL_READ)
+        assert np.array_equal(yh, eval_f1.saxpy(y0, xh, -0.75))
+    finally:
+        hpl.hpl_array_free(x)
+        hpl.hpl_array_free(y)
