@@ -35,6 +35,9 @@ evalab)
   for v in ${EVV}; do echo "== $v" >> gpurun_out/${TAG}_evalab.jsonl; HPL_LIB=$PWD/ab_ship/libhpl_$v.so timeout 300 python tools/bench_eval.py >> gpurun_out/${TAG}_evalab.jsonl 2>&1; done
   HPL_LIB=$PWD/ab_ship/libhpl_${PTV}.so timeout 600 python -m pytest tests/test_eval.py -m gpu -q > gpurun_out/${TAG}_evaltests.log 2>&1; tail -2 gpurun_out/${TAG}_evaltests.log
   grep -v saxpy gpurun_out/${TAG}_evalab.jsonl | cut -c1-160 ;;
+spmvab)
+  for v in ${SPV}; do echo "== $v" >> gpurun_out/${TAG}_spmv.jsonl; HPL_LIB=$PWD/ab_ship/libhpl_$v.so timeout 300 python tools/bench_spmv.py >> gpurun_out/${TAG}_spmv.jsonl 2>&1; done
+  HPL_LIB=$PWD/ab_ship/libhpl_${PTV}.so timeout 600 python -m pytest tests/test_spmv.py -m gpu -q > gpurun_out/${TAG}_spmvtests.log 2>&1; tail -2 gpurun_out/${TAG}_spmvtests.log ;;
 ref)
   timeout 600 python bench.py --impl reference > gpurun_out/${TAG}_ref.json 2> gpurun_out/${TAG}_ref.err; cat gpurun_out/${TAG}_ref.json ;;
 ab)
