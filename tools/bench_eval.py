@@ -61,7 +61,7 @@ timed("saxpy", [y, x], [y, x, 1.5], [n], None, 24 * n)
 hpl.hpl_array_free(y); hpl.hpl_array_free(x)
 
 # dotp (Fig. 4): v1, v2 f32, pSums one per group of M
-for M in (32, 64, 128, 256, 1024):
+for M in [int(x) for x in os.environ.get("EVAL_MS", "32,64,128,256,1024").split(",")]:
     v1 = hpl.hpl_array_alloc(hpl.HPL_F32, [n])
     v2 = hpl.hpl_array_alloc(hpl.HPL_F32, [n])
     ps = hpl.hpl_array_alloc(hpl.HPL_F32, [n // M])
