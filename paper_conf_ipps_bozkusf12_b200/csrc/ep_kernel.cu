@@ -1267,17 +1267,26 @@ static EPKernel tier_kernel(int thr) {
 #define EP_T256_W EP_ILP
 #endif
 #ifndef EP_T384_MINB
-#define EP_T384_MINB 2
+#define EP_T384_MINB 1   // one CTA per SM (the 139-KB table allows no second one): up to 170 registers
 #endif
 #ifndef EP_T384_W
-#define EP_T384_W EP_ILP
+#define EP_T384_W 4      // 140 registers, no spills; the default tier (EP_DEFAULT_THREADS)
+#endif
+#ifndef EP_TIER_X
+#define EP_TIER_X 0    // an extra launch-bound tier between 384 and 512 threads (0: none)
+#endif
+#ifndef EP_TIER_X_W
+#define EP_TIER_X_W 4
 #endif
 #ifndef EP_T512_W
 #define EP_T512_W 3  // 120 registers, no spills (round 2: W = 2 is 4 % slower, W = 4 spills)
 #endif
   if (thr <= 128) return ep_kernel<V, A32, 128, 4, 1>;   // 128 regs
   if (thr <= 256) return ep_kernel<V, A32, 256, EP_T256_MINB, EP_T256_W>;   //  85 regs (3 blocks/SM)
-  if (thr <= 384) return ep_kernel<V, A32, 384, EP_T384_MINB, EP_T384_W>;   //  85 regs (2 blocks/SM)
+  if (thr <= 384) return ep_kernel<V, A32, 384, EP_T384_MINB, EP_T384_W>;   // 140 regs, W = 4 (default)
+#if EP_TIER_X
+  if (thr <= EP_TIER_X) return ep_kernel<V, A32, EP_TIER_X, 1, EP_TIER_X_W>;  // extra tier (A/B)
+#endif
   if (thr <= 512) return ep_kernel<V, A32, 512, 1, EP_T512_W>;   // 128 regs
   if (thr <= 640) return ep_kernel<V, A32, 640, 1, EP_ILP>;   // 102 regs
   if (thr <= 768) return ep_kernel<V, A32, 768, 1, EP_ILP>;   //  85 regs
@@ -1394,7 +1403,7 @@ int set_attrs_once(int device) {
   if ((int)done.size() <= device) done.resize(device + 1, 0);
   if (done[device]) return 0;
   const int smem = int(LOG_TAB * sizeof(LogEntry));
-  for (int thr : {128, 256, 384, 512, 640, 768, 1024})
+  for (int thr : {128, 256, 384, EP_TIER_X ? EP_TIER_X : 512, 512, 640, 768, 1024})
     for (bool a32 : {true, false}) {
       cudaError_t e = cudaFuncSetAttribute(pick_kernel(HPL_VARIANT_LEAN, a32, thr),
                                            cudaFuncAttributeMaxDynamicSharedMemorySize, smem);

@@ -12,7 +12,10 @@ namespace hplep {
 
 constexpr int HPL_VARIANT_LEAN = HPL_EP_LEAN;
 constexpr int HPL_VARIANT_LIBDEVICE = HPL_EP_LIBDEVICE;
-constexpr int EP_DEFAULT_THREADS = 512;
+#ifndef EP_DEFAULT_THREADS_CFG
+#define EP_DEFAULT_THREADS_CFG 384  // 12 warps x 4 pairs in lockstep (round 2: +2.1 % over 16 warps x 3)
+#endif
+constexpr int EP_DEFAULT_THREADS = EP_DEFAULT_THREADS_CFG;
 #ifndef EP_MIN_PPT
 #define EP_MIN_PPT 8   // min pairs per thread before the grid grows (64 -> 8: -8 us at 2^16 pairs, session 3)
 #endif

@@ -24,8 +24,8 @@ def one(spec):
                        capture_output=True, text=True)
     if r.returncode:
         return name, "BUILD FAILED " + r.stderr[-400:]
-    pat = os.environ.get("MG_PAT", "ILi0ELb1ELi512ELi1ELi3E")
-    ppi = os.environ.get("MG_PPI", "6")
+    pat = os.environ.get("MG_PAT", "ILi0ELb1ELi384ELi1ELi4E")
+    ppi = os.environ.get("MG_PPI", "16")
     o = subprocess.run([sys.executable, os.path.join(ROOT, "tools", "sass_hot.py"), cub, pat, ppi],
                        capture_output=True, text=True).stdout.splitlines()
     return name, " | ".join(x.strip() for x in o[:3])

@@ -16,8 +16,8 @@ import subprocess
 import sys
 
 lib = sys.argv[1] if len(sys.argv) > 1 else "paper_conf_ipps_bozkusf12_b200/libhpl.so"
-pat = sys.argv[2] if len(sys.argv) > 2 else "ILi0ELb1ELi512ELi1ELi3E"
-ppi = int(sys.argv[3]) if len(sys.argv) > 3 else 6
+pat = sys.argv[2] if len(sys.argv) > 2 else "ILi0ELb1ELi384ELi1ELi4E"
+ppi = int(sys.argv[3]) if len(sys.argv) > 3 else 16
 out = subprocess.run(["cuobjdump", "-sass", lib], capture_output=True, text=True).stdout
 ins, on = [], False
 for ln in out.splitlines():

@@ -1,6 +1,6 @@
 """Print the hot loop as a string of F (FP64) / i (other) and run statistics."""
 import re, subprocess, sys, collections
-lib = sys.argv[1]; pat = sys.argv[2] if len(sys.argv) > 2 else "ILi0ELb1ELi512ELi1ELi3E"
+lib = sys.argv[1]; pat = sys.argv[2] if len(sys.argv) > 2 else "ILi0ELb1ELi384ELi1ELi4E"
 out = subprocess.run(["cuobjdump", "-sass", lib], capture_output=True, text=True).stdout
 ins, on = [], False
 for ln in out.splitlines():
