@@ -66,7 +66,7 @@ __device__ __forceinline__ double rsqrt_approx(double p) {
 #define EP_TICKET_ACQ 1  // 1: last-block detection by an acquiring ticket atomic instead of a second fence (-0.3 us)
 #endif
 #ifndef EP_IDX_ONE
-#define EP_IDX_ONE 0  // 1: the +1 of the fused-t' index from a loop-invariant register (-0.33 IMAD.MOV/pair; measured -2.7 %)
+#define EP_IDX_ONE 1  // 1: the +1 of the fused-t' index from a loop-invariant register (-0.33 IMAD.MOV/pair: +1.6 % with the 384 x 4 default, -2.7 % with 512 x 3)
 #endif
 __device__ __forceinline__ unsigned tab_addr(unsigned H, unsigned tabb, unsigned one = 1u) {
 #if EP_IDX_TRUNC && EP_T_FMA == 2 && EP_IDX_ONE
