@@ -93,6 +93,7 @@ class ClockSampler:
         self.index = index
         self.rows = []
         self.proc = None
+        self.t0 = None
 
     def start(self):
         try:
@@ -109,7 +110,13 @@ class ClockSampler:
         for line in self.proc.stdout:
             parts = [x.strip() for x in line.split(",")]
             if len(parts) == 7:
-                self.rows.append(parts)
+                self.rows.append((time.time(), parts))
+
+    def mark(self):
+        """Start of the timed region: nvidia-smi was started before the
+        warm-up (its NVML start-up would otherwise land in the first timed
+        step), and only samples from here on count."""
+        self.t0 = time.time()
 
     def stop(self):
         if self.proc is None:
@@ -119,7 +126,7 @@ class ClockSampler:
             self.proc.wait(timeout=5)
         except Exception:
             self.proc.kill()
-        rows = self.rows
+        rows = [r for t, r in self.rows if self.t0 is None or t >= self.t0] or [r for _, r in self.rows]
         names = ["sw_power_cap", "hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown"]
         sm = [float(r[0]) for r in rows if r[0].replace(".", "").isdigit()]
         mx = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
@@ -290,6 +297,8 @@ def run_ours(args, M):
         else:
             hpl.hpl_ep_run_shard(M, NPB_SEED, NPB_A, rank, world, out.data_ptr(), stream.cuda_stream)
 
+    sampler = ClockSampler(gpu)
+    sampler.start()
     for _ in range(args.warmup):
         step()
         if combine == "nccl":
@@ -317,11 +326,10 @@ def run_ours(args, M):
             torch.cuda.synchronize(dev)
 
     # ---- device-timed region
-    sampler = ClockSampler(gpu)
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize(dev)
-    sampler.start()
+    sampler.mark()
     launches0 = hpl.hpl_ep_launch_count()
     step_ms, kern_ms = [], []
     for _ in range(args.steps):
