@@ -31,6 +31,16 @@ EP_HD uint64_t state_to_v(uint64_t x) { return EXP_ONE | (x << 6); }
 EP_HD uint64_t v_to_state(uint64_t v) { return (v & MASK52) >> 6; }
 EP_HD uint64_t step_v(uint64_t v, uint64_t a) { return ((a * v) & MASK52) | EXP_ONE; }
 
+// The I2F form (EP_I2F, the default): y = x 2^18 - 2^63 as a signed 64-bit
+// integer, i.e. the state in the top 46 bits with the sign bit flipped.  For
+// odd a, a (y + 2^63) + 2^63 = a y + (a + 1) 2^63 = a y (mod 2^64), so one LCG
+// step is y' = a y mod 2^64 (two integer instructions, the low 18 bits stay
+// 0), and the exact conversion I2F.F64.S64(y) = (x - 2^45) 2^18 = x' 2^64 is
+// NPB's x/2 = u - 1/2 scaled by a power of two.
+constexpr uint64_t SIGN64 = uint64_t(1) << 63;
+EP_HD uint64_t state_to_y(uint64_t x) { return (x << 18) ^ SIGN64; }
+EP_HD uint64_t y_to_state(uint64_t y) { return (y ^ SIGN64) >> 18; }
+
 // Jump table J[i] = a^(2^i) mod 2^46, i = 0..45.
 constexpr int NJUMP = 46;
 

@@ -56,6 +56,14 @@ __device__ __forceinline__ double rsqrt_approx(double p) {
 #ifndef EP_LCG_CARRY
 #define EP_LCG_CARRY 1  // 1: LCG carries the unmasked high word (IMAD reads one odd register)
 #endif
+#ifndef EP_I2F
+#define EP_I2F 0        // 1: x'' = I2F.F64.S64(y) = x' 2^64 from the signed LCG state (no LOP3, no DADD map);
+#endif                  //    t'' = t' 2^128, table inverses scaled by 2^-128.  18 FP64/pair
+                        //    and parity green, but 9 % slower at class D (1.155 vs 1.273 M, r02aj): the
+                        //    64-bit-source conversion costs ~7 issue cycles per warp instruction here
+// t'' = t' * 2^EP_TSH and x'' = x' * 2^(EP_TSH/2) (exact power-of-two scalings of NPB's roundings)
+constexpr unsigned EP_TSH = EP_I2F ? 128u : 0u;
+constexpr double EP_TSCALE = EP_I2F ? 0x1p128 : 1.0;
 #ifndef EP_E_SQ
 #define EP_E_SQ 1       // 1: Newton residual e = 1 - p y0^2 with y0^2 exact (one register pair)
 #endif
@@ -70,12 +78,12 @@ __device__ __forceinline__ double rsqrt_approx(double p) {
 #endif
 __device__ __forceinline__ unsigned tab_addr(unsigned H, unsigned tabb, unsigned one = 1u) {
 #if EP_IDX_TRUNC && EP_T_FMA == 2 && EP_IDX_ONE
-  return ((max(H + one, TRUNC_HLO) >> LOG_SHIFT) << 4) + tabb;
+  return ((max(H + one, TRUNC_HLO + (EP_TSH << 20)) >> LOG_SHIFT) << 4) + tabb;
 #elif EP_IDX_TRUNC && EP_T_FMA == 2
   // H + 1: the fused t' with high word 0x3FCFFFFF (just below 1/4) shares the
   // NaN bucket of [1/4, 1/4 + w) -> rare path (exact acceptance); other t'
   // move at most one high-word step (|r| <= 2^-10 + 2^-20)
-  return ((max(H + 1u, TRUNC_HLO) >> LOG_SHIFT) << 4) + tabb;
+  return ((max(H + 1u, TRUNC_HLO + (EP_TSH << 20)) >> LOG_SHIFT) << 4) + tabb;
 #elif EP_IDX_TRUNC
   return ((max(H, TRUNC_HLO) >> LOG_SHIFT) << 4) + tabb;
 #else
@@ -84,11 +92,12 @@ __device__ __forceinline__ unsigned tab_addr(unsigned H, unsigned tabb, unsigned
 }
 __device__ __forceinline__ unsigned tab_base(const void* smem) {
   const unsigned b = static_cast<unsigned>(__cvta_generic_to_shared(smem));
-  return EP_IDX_TRUNC ? b - TRUNC_J0 * 16u : b;
+  // (the t'' scaling moves every index by EP_TSH << LOG_K entries: folded into the base)
+  return EP_IDX_TRUNC ? b - (TRUNC_J0 + (EP_TSH << LOG_K)) * 16u : b;
 }
 // t' below the table (truncating mode; the exact rare path recomputes these pairs)
 __device__ __forceinline__ bool below_table(double t) {
-  return static_cast<unsigned>(__double2hiint(t)) < (LOG_IDX_MIN << LOG_SHIFT);
+  return static_cast<unsigned>(__double2hiint(t)) < (LOG_IDX_MIN << LOG_SHIFT) + (EP_TSH << 20);
 }
 
 #ifndef EP_Y0LO
@@ -185,6 +194,27 @@ __device__ __forceinline__ void lcg_step_c(unsigned& lo, unsigned& ph, unsigned&
   asm("lop3.b32 %0, %1, 0x000FFFFF, %2, 0xEA;" : "=r"(hd) : "r"(ph), "r"(exp_hi));
 }
 
+// I2F form (ep_common.cuh state_to_y): y' = a y mod 2^64 = IMAD.WIDE.U32 + IMAD
+// (+ IMAD if a >= 2^32); the uniform is then one exact I2F.F64.S64.
+template <bool A32>
+__device__ __forceinline__ void lcg_step_y(unsigned& lo, unsigned& hi, unsigned a_lo, unsigned a_hi) {
+#ifndef EP_Y64
+#define EP_Y64 0  // 1: one 64-bit multiply (ptxas: IMAD.WIDE.U32 into the state pair + IMAD on its high word)
+#endif
+  if (EP_Y64) {
+    uint64_t y = (static_cast<uint64_t>(hi) << 32) | lo;
+    y *= A32 ? static_cast<uint64_t>(a_lo) : ((static_cast<uint64_t>(a_hi) << 32) | a_lo);
+    lo = static_cast<unsigned>(y);
+    hi = static_cast<unsigned>(y >> 32);
+  } else {
+    hi = __umulhi(lo, a_lo) + hi * a_lo + (A32 ? 0u : lo * a_hi);
+    lo = lo * a_lo;
+  }
+}
+__device__ __forceinline__ double y_to_x2(unsigned lo, unsigned hi) {  // x'' = x' 2^64, exact
+  return __ll2double_rn(static_cast<long long>((static_cast<uint64_t>(hi) << 32) | lo));
+}
+
 template <bool A32>
 __device__ __forceinline__ void lcg_step(unsigned& lo, unsigned& hi, unsigned a_lo, unsigned a_hi) {
   const unsigned ph = __umulhi(lo, a_lo) + hi * a_lo + (A32 ? 0u : lo * a_hi);
@@ -246,7 +276,7 @@ __device__ __noinline__ RareOut rare_pair(double t, double x1, double x2, double
 #else
   const double tf = t;
 #endif
-  if (t > 0.25) return RareOut{0.0, 0.0, 0u};  // rejected
+  if (t > 0.25 * EP_TSCALE) return RareOut{0.0, 0.0, 0u};  // rejected
 #if EP_IDX_TRUNC
   (void)u;
   if (below_table(t) || t != tf || X != X) {  // (NaN: EP_T_FMA == 2's bucket at 1/4)
@@ -255,10 +285,10 @@ __device__ __noinline__ RareOut rare_pair(double t, double x1, double x2, double
   if (u >= LOG_N || t != tf) {
 #endif  // t below the table: NPB's formula, libdevice log/sqrt, on
     // the unscaled t = 4 t', x = 2 x' (exact)
-    const double tt = 4.0 * t;
+    const double tt = (4.0 / EP_TSCALE) * t;
     const double t2 = sqrt(-2.0 * log(tt) / tt);
-    X = __dmul_rn(2.0 * x1, t2);
-    Y = __dmul_rn(2.0 * x2, t2);
+    X = __dmul_rn((EP_I2F ? 0x1p-63 : 2.0) * x1, t2);
+    Y = __dmul_rn((EP_I2F ? 0x1p-63 : 2.0) * x2, t2);
   }
   const unsigned l = __double2uint_rz(fmax(fabs(X), fabs(Y)));
   RareOut o{X, Y, 0u};
@@ -494,6 +524,9 @@ constexpr int EP_WIN_N = (NJUMP + 3) / 4;  // 12 windows cover 2 p0 < 2^46
 #ifndef EP_PIPE
 #define EP_PIPE 1      // 1: software-pipeline generation of group g+1 under the transform of group g
 #endif
+#if EP_I2F && !(EP_IDX_TRUNC && EP_T_FMA == 2 && EP_ACC_HI && EP_PRED_MODE == 0 && EP_PIPE && !EP_MAXSQ && !EP_LCG_PAR)
+#error "EP_I2F is built for the default pipelined path (truncating index, fused t', high-word acceptance)"
+#endif
 
 // Software-pipelined form of lean_pairs: gen_stage produces the LCG pairs, t',
 // the table index and the table entries of a group (integer + LDS heavy);
@@ -511,6 +544,13 @@ __device__ __forceinline__ void gen_stage(unsigned& vlo, unsigned& vhi, const EP
                                           Stage<W>& S, unsigned exp_hi, unsigned one = 1u) {
 #pragma unroll
   for (int k = 0; k < W; ++k) {
+#if EP_I2F && !(EP_ABL & 2)
+    lcg_step_y<A32>(vlo, vhi, P.a_lo, P.a_hi);
+    S.x1[k] = y_to_x2(vlo, vhi);
+    lcg_step_y<A32>(vlo, vhi, P.a_lo, P.a_hi);
+    S.x2[k] = y_to_x2(vlo, vhi);
+    (void)exp_hi;
+#else
 #if EP_ABL & 2  // ablation (timing only, wrong results): LCG step -> one add
     vlo += P.a_lo;
 #elif EP_LCG_CARRY
@@ -533,6 +573,7 @@ __device__ __forceinline__ void gen_stage(unsigned& vlo, unsigned& vhi, const EP
 #endif
 #if !EP_LCG_CARRY || (EP_ABL & 2)
     S.x2[k] = __dadd_rn(__hiloint2double(int(vhi), int(vlo)), -1.5);
+#endif
 #endif
   }
 #pragma unroll
@@ -595,7 +636,7 @@ __device__ __forceinline__ void transform_stage(const Stage<W>& S, const EPParam
       // t' == 1/4 (L = 0 -> X = Y = 0, bin 0: correct on the fast path) and
       // rejects just above 1/4, whose L < 0 makes X, Y NaN -> selector says
       // "rare" -> rare_pair rejects them exactly (t > 0.25)
-      acc[k] = static_cast<unsigned>(__double2hiint(S.t[k])) <= 0x3FD00000u;
+      acc[k] = static_cast<unsigned>(__double2hiint(S.t[k])) <= 0x3FD00000u + (EP_TSH << 20);
     else if (EP_ACC_INT)
       acc[k] = static_cast<unsigned long long>(__double_as_longlong(S.t[k])) <= 0x3FD0000000000000ull;
     else
@@ -712,10 +753,10 @@ __device__ __forceinline__ void transform_stage(const Stage<W>& S, const EPParam
     }
     if (DBG) {  // test hook (hpl_ep_pairs_debug): t, X, Y, l (-1 rare path, -2 rejected)
       // t as NPB rounds it (the fused t' of EP_T_FMA is internal)
-      dbg[4 * k + 0] = 4.0 * __dadd_rn(__dmul_rn(S.x1[k], S.x1[k]), __dmul_rn(S.x2[k], S.x2[k]));
+      dbg[4 * k + 0] = (4.0 / EP_TSCALE) * __dadd_rn(__dmul_rn(S.x1[k], S.x1[k]), __dmul_rn(S.x2[k], S.x2[k]));
       dbg[4 * k + 1] = ok[k] ? X[k] : 0.0;
       dbg[4 * k + 2] = ok[k] ? Y[k] : 0.0;
-      const bool acc_npb = __dadd_rn(__dmul_rn(S.x1[k], S.x1[k]), __dmul_rn(S.x2[k], S.x2[k])) <= 0.25;
+      const bool acc_npb = __dadd_rn(__dmul_rn(S.x1[k], S.x1[k]), __dmul_rn(S.x2[k], S.x2[k])) <= 0.25 * EP_TSCALE;
       dbg[4 * k + 3] = !acc_npb ? -2.0 : ok[k] ? double(EP_BIN_MODE == 3 ? l[k] & 3u : l[k]) : -1.0;
     }
   }
@@ -769,7 +810,8 @@ __global__ void __launch_bounds__(256) ep_pairs_debug_kernel(const __grid_consta
   if (i >= n) return;
   const unsigned tab = tab_base(smem_raw);
   const LeanConst K = make_lean_const(static_cast<unsigned>(__cvta_generic_to_shared(s_kc)));
-  const uint64_t v0 = state_to_v(jump_state(P.x_begin, 2 * i, P.jump));
+  const uint64_t x0 = jump_state(P.x_begin, 2 * i, P.jump);
+  const uint64_t v0 = EP_I2F ? state_to_y(x0) : state_to_v(x0);
   unsigned vlo = unsigned(v0), vhi = unsigned(v0 >> 32);
   Stage<1> S;
   gen_stage<A32, 1>(vlo, vhi, P, tab, S, K.exp_hi);
@@ -970,7 +1012,7 @@ ep_kernel(const __grid_constant__ EPParams P) {
 #pragma unroll 1
   for (uint64_t k = 2 * p0, wi = 0; k != 0; k >>= 4, ++wi)
     if (k & 15) xj = mulmod46(xj, s_win[wi][k & 15]);
-  const uint64_t v0 = state_to_v(xj);
+  const uint64_t v0 = (EP_I2F && VARIANT == HPL_VARIANT_LEAN && EP_PIPE) ? state_to_y(xj) : state_to_v(xj);
 #else
   const uint64_t v0 = state_to_v(jump_state(P.x_begin, 2 * p0, P.jump));
 #endif
@@ -1242,9 +1284,16 @@ __global__ void lcg_states_kernel(uint64_t seed, uint64_t a, uint64_t offset, ui
                                   const __grid_constant__ JumpTable J, uint64_t* out) {
   const uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
   if (i >= n) return;
+  const unsigned a_lo = unsigned(a), a_hi = unsigned(a >> 32), exp_hi = 0x3FF00000u;
+#if EP_I2F
+  const uint64_t y = state_to_y(jump_state(seed, offset + i, J.j));
+  unsigned lo = unsigned(y), hi = unsigned(y >> 32);
+  lcg_step_y<A32>(lo, hi, a_lo, a_hi);
+  (void)exp_hi;
+  out[i] = y_to_state((uint64_t(hi) << 32) | lo);
+#else
   const uint64_t v = state_to_v(jump_state(seed, offset + i, J.j));
   unsigned lo = unsigned(v), hi = unsigned(v >> 32), hd;
-  const unsigned a_lo = unsigned(a), a_hi = unsigned(a >> 32), exp_hi = 0x3FF00000u;
 #if EP_LCG_CARRY
   lcg_step_c<A32>(lo, hi, hd, a_lo, a_hi, exp_hi);
 #else
@@ -1252,6 +1301,7 @@ __global__ void lcg_states_kernel(uint64_t seed, uint64_t a, uint64_t offset, ui
   hd = hi;
 #endif
   out[i] = v_to_state((uint64_t(hd) << 32) | lo);
+#endif
 }
 
 // ------------------------------------------------------------- dispatcher
@@ -1347,7 +1397,7 @@ void build_log_table(std::vector<LogEntry>& tab) {
       const long double centre =
           ldexpl(1.0L + ((long double)(j & ((1u << LOG_K) - 1)) + 0.5L) / (1 << LOG_K), E);
       const float inv = (float)(1.0L / centre);
-      tab[e].inv = (double)inv;
+      tab[e].inv = ldexp((double)inv, -int(EP_TSH));  // (t'' = t' 2^EP_TSH: r = t'' inv'' - 1 unchanged)
       tab[e].T = (double)(2.0L * logl((long double)inv * 0.25L));  // -2 ln(4 t') at r = 0
     } else if (EP_T_FMA == 2 && j == LOG_IDX_MAX) {  // [1/4, 1/4 + w) and, via the H + 1 index,
       tab[e].T = __builtin_nan("");                  // the fused t' just below 1/4: NaN -> the
@@ -1356,9 +1406,9 @@ void build_log_table(std::vector<LogEntry>& tab) {
                                         // r = 4t' - 1 exact): L = -2 ln(1 + r) has no cancellation
                                         // as t' -> 1/4; t' = 1/4 -> L = 0; above -> L < 0 -> NaN
       tab[e].T = 0.0;
-      tab[e].inv = 4.0;
-    } else {                            // reject sentinels up to t' = 1/2
-      tab[e].T = 0x1p1000;
+      tab[e].inv = ldexp(4.0, -int(EP_TSH));
+    } else {                            // reject sentinels up to t' = 1/2 (L t'' stays finite)
+      tab[e].T = EP_I2F ? 0x1p800 : 0x1p1000;
       tab[e].inv = 0.0;
     }
   }

@@ -42,6 +42,11 @@ __global__ void __launch_bounds__(512, 1) k(double* out, unsigned* iout, long lo
         if (OP == 14) { double y; asm volatile("rsqrt.approx.ftz.f64 %0, %1;" : "=d"(y) : "d"(__hiloint2double(int(u[i]), 0))); u[i] = unsigned(__double2hiint(y)); }
         if (OP == 15) asm volatile("fma.rn.f32 %0, %0, %1, 0f3F800000;" : "+f"(g[i]) : "f"(g[(i + 1) & 7]));
         if (OP == 16) asm volatile("min.u32 %0, %0, 0x2001;" : "+r"(u[i]));
+        if (OP == 17) asm volatile("{.reg .f64 t; cvt.rn.f64.s64 t, %0; mov.b64 %0, t;}" : "+l"(q[i]));
+        if (OP == 18) asm volatile("add.rn.f64 %0, %0, %1;" : "+d"(e[i]) : "d"(f[(i + 1) & 7]));
+        if (OP == 19) asm volatile("{.reg .f64 t; cvt.rn.f64.u32 t, %0; mov.b64 %1, t;}" : "+r"(u[i]), "+l"(q[i]));
+        if (OP == 20) { asm volatile("lop3.b32 %0, %0, 0xfffff, %1, 0xea;" : "+r"(u[i]) : "r"(w[i]));
+                        asm volatile("add.rn.f64 %0, %0, %1;" : "+d"(e[i]) : "d"(f[(i + 1) & 7])); }
       }
     }
   }
@@ -88,5 +93,9 @@ int main() {
   RUN(13, "F2I.U32.F64");
   RUN(14, "MUFU.RSQ64H");
   RUN(15, "FFMA");
+  RUN(17, "I2F.F64.S64");
+  RUN(18, "DADD R,R");
+  RUN(19, "I2F.F64.U32");
+  RUN(20, "LOP3+DADD");
   return 0;
 }
